@@ -1,0 +1,55 @@
+"""Mutation check for the oracle pins: apply one plausible mistake at a time to oracle/ and
+confirm that `pytest tests/test_oracle_*.py` fails.  Usage: python tools/mutate_oracle.py"""
+import os
+import shutil
+import subprocess
+import sys
+import tempfile
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+MUTANTS = [
+    ("oracle/kv.py", "return s * g.slab_bytes + l * k * Cl + j * Cl", "return s * g.slab_bytes + j * k * Cl + l * Cl"),
+    ("oracle/kv.py", "return s * g.slab_bytes + j * L * Cl + l * Cl", "return s * g.slab_bytes + l * L * Cl + j * Cl"),
+    ("oracle/kv.py", "d = ((l - l0) * n + i) * c\n            stage[d:d + c]", "d = (i * (l1 - l0) + (l - l0)) * c\n            stage[d:d + c]"),
+    ("oracle/kv.py", "out[a:a + c] = stage[d:d + c]", "out[a:a + c] = stage[d:d + c][::-1]"),
+    ("oracle/kv.py", "out = dst.copy()", "out = np.zeros_like(dst)"),
+    ("oracle/shape.py", "return self.L * 2 * self.H * self.D * self.s", "return self.L * self.H * self.D * self.s"),
+    ("oracle/shape.py", "return (((c * self.B + slot) * self.H + h) * self.D + d) * self.s", "return (((c * self.B + h) * self.H + slot) * self.D + d) * self.s"),
+    ("oracle/slab.py", "if j not in self.owned[s] and (s, j) not in self.quarantine:", "if j not in self.owned[s]:"),
+    ("oracle/slab.py", "for s in range(self.n_slabs):\n            if self.shape[s] is not None:", "for s in reversed(range(self.n_slabs)):\n            if self.shape[s] is not None:"),
+    ("oracle/slab.py", "if busy:\n                self.quarantine[(s, j)] = busy", "if False:\n                self.quarantine[(s, j)] = busy"),
+    ("oracle/slab.py", "                self.shape[s] = None\n", "                pass\n"),
+    ("oracle/slab.py", "return self.slab_bytes // shape.block_bytes()", "return -(-self.slab_bytes // shape.block_bytes())"),
+    ("oracle/weights.py", "return w[:, r * part:(r + 1) * part]", "return w[:, r:(r + 1) * part]"),
+    ("oracle/weights.py", "for gi in range(groups)], axis=0)", "for gi in range(groups)][::-1], axis=0)"),
+    ("oracle/weights.py", "p = align_up(p + n)", "p = p + n"),
+    ("oracle/rules.py", "pending.setdefault(e[1], set()).add(c)", "pass"),
+    ("oracle/rules.py", "captured[e[2]] = tail.get(e[1])", "captured[e[2]] = len(ops) - 1 if ops else None"),
+]
+
+
+def main():
+    survived = []
+    for path, old, new in MUTANTS:
+        with tempfile.TemporaryDirectory() as d:
+            for sub in ("oracle", "tests", "aeg_inputs"):
+                shutil.copytree(os.path.join(ROOT, sub), os.path.join(d, sub),
+                                ignore=shutil.ignore_patterns("__pycache__", "*.so"))
+            f = os.path.join(d, path)
+            src = open(f).read()
+            assert old in src, (path, old)
+            open(f, "w").write(src.replace(old, new, 1))
+            r = subprocess.run([sys.executable, "-m", "pytest", "-x", "-q", "-p", "no:cacheprovider",
+                                "tests/test_oracle_shape.py", "tests/test_oracle_slab.py", "tests/test_oracle_kv.py",
+                                "tests/test_oracle_weights.py", "tests/test_oracle_rules.py"],
+                               cwd=d, capture_output=True, text=True)
+            status = "killed" if r.returncode != 0 else "SURVIVED"
+            print(f"{status:9s} {path}: {new[:70]!r}")
+            if r.returncode == 0:
+                survived.append((path, new))
+    print(f"{len(MUTANTS) - len(survived)}/{len(MUTANTS)} mutants killed")
+    return 1 if survived else 0
+
+
+if __name__ == "__main__":
+    sys.exit(main())
