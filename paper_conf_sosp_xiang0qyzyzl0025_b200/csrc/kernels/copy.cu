@@ -1,0 +1,241 @@
+// Block-table copy kernels for B200 (sm_100a).  See copy.h for the addressing contract.
+//
+// Two implementations of the same byte copy, selected by measurement:
+//  * LSU  : 256-thread CTAs; a work item is a 32 KiB piece of one (block, layer) chunk; each
+//           thread issues 8 independent 16-byte ld.global.nc.L1::no_allocate (all loads first,
+//           then all stores) so ~128 KiB per SM are in flight; the block-table entry of an item
+//           is one broadcast load per warp.
+//  * BULK : the Blackwell async path: one thread per CTA drives a STAGES-deep ring of PIECE-byte
+//           shared-memory buffers with cp.async.bulk (global->smem, mbarrier complete_tx) and
+//           cp.async.bulk (smem->global, bulk_group); no data passes through registers.
+// Both are persistent: the grid is one wave (148 SMs x resident CTAs) striding over items.
+#include <cuda_runtime.h>
+
+#include <cstdint>
+
+#include "copy.h"
+
+namespace aeg {
+namespace {
+
+constexpr int kSMs = 148;
+
+__device__ __forceinline__ uint4 ld_stream(const void* p) {
+  uint4 v;
+  asm volatile("ld.global.nc.L1::no_allocate.v4.u32 {%0,%1,%2,%3}, [%4];"
+               : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w)
+               : "l"(p));
+  return v;
+}
+
+__device__ __forceinline__ void st_stream(void* p, const uint4& v) {
+  asm volatile("st.global.L1::no_allocate.v4.u32 [%0], {%1,%2,%3,%4};" ::"l"(p), "r"(v.x), "r"(v.y), "r"(v.z),
+               "r"(v.w)
+               : "memory");
+}
+
+template <bool SP, bool DP>
+__device__ __forceinline__ void item_ptrs(const CopyArgs& a, uint64_t c, const char*& s, char*& d) {
+  const uint32_t t = uint32_t(c / uint64_t(a.n));
+  const uint32_t i = uint32_t(c - uint64_t(t) * a.n);
+  if (SP)
+    s = a.src + __ldg(a.src_off + i) + uint64_t(a.l_first + t) * a.src_lstride;
+  else
+    s = a.src + c * a.chunk;  // (t * n + i) * chunk
+  if (DP)
+    d = a.dst + __ldg(a.dst_off + i) + uint64_t(a.l_first + t) * a.dst_lstride;
+  else
+    d = a.dst + c * a.chunk;
+}
+
+// ------------------------------------------------------------------------------------- LSU
+constexpr int kLsuThreads = 256;
+constexpr int kLsuUnroll = 8;
+constexpr uint64_t kLsuPiece = uint64_t(kLsuThreads) * 16 * kLsuUnroll;  // 32 KiB
+
+template <bool SP, bool DP>
+__global__ void __launch_bounds__(kLsuThreads) copy_lsu(const CopyArgs a) {
+  const uint64_t ppc = (a.chunk + kLsuPiece - 1) / kLsuPiece;
+  const uint64_t items = uint64_t(a.nl) * uint64_t(a.n) * ppc;
+  for (uint64_t w = blockIdx.x; w < items; w += gridDim.x) {
+    const uint64_t c = w / ppc;
+    const uint64_t base = (w - c * ppc) * kLsuPiece;
+    const char* s;
+    char* d;
+    item_ptrs<SP, DP>(a, c, s, d);
+    uint4 v[kLsuUnroll];
+    if (base + kLsuPiece <= a.chunk) {
+#pragma unroll
+      for (int u = 0; u < kLsuUnroll; ++u) v[u] = ld_stream(s + base + (uint64_t(u) * kLsuThreads + threadIdx.x) * 16);
+#pragma unroll
+      for (int u = 0; u < kLsuUnroll; ++u) st_stream(d + base + (uint64_t(u) * kLsuThreads + threadIdx.x) * 16, v[u]);
+    } else {
+#pragma unroll
+      for (int u = 0; u < kLsuUnroll; ++u) {
+        const uint64_t o = base + (uint64_t(u) * kLsuThreads + threadIdx.x) * 16;
+        if (o < a.chunk) v[u] = ld_stream(s + o);
+      }
+#pragma unroll
+      for (int u = 0; u < kLsuUnroll; ++u) {
+        const uint64_t o = base + (uint64_t(u) * kLsuThreads + threadIdx.x) * 16;
+        if (o < a.chunk) st_stream(d + o, v[u]);
+      }
+    }
+  }
+}
+
+// ------------------------------------------------------------------------------------ BULK
+constexpr int kBulkStages = 6;
+constexpr uint32_t kBulkPiece = 32768;
+constexpr int kBulkSmem = kBulkStages * kBulkPiece;  // 192 KiB -> one CTA per SM
+
+__device__ __forceinline__ uint32_t smem_u32(const void* p) {
+  return static_cast<uint32_t>(__cvta_generic_to_shared(p));
+}
+
+__device__ __forceinline__ void mbar_init(uint64_t* bar, uint32_t count) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count) : "memory");
+}
+
+__device__ __forceinline__ void bulk_load(void* sdst, const void* gsrc, uint32_t bytes, uint64_t* bar) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(bytes)
+               : "memory");
+  asm volatile(
+      "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+          smem_u32(sdst)),
+      "l"(gsrc), "r"(bytes), "r"(smem_u32(bar))
+      : "memory");
+}
+
+__device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t phase) {
+  asm volatile(
+      "{\n"
+      ".reg .pred p;\n"
+      "WAIT_%=:\n"
+      "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n"
+      "@!p bra WAIT_%=;\n"
+      "}\n" ::"r"(smem_u32(bar)),
+      "r"(phase)
+      : "memory");
+}
+
+__device__ __forceinline__ void bulk_store(void* gdst, const void* ssrc, uint32_t bytes) {
+  asm volatile("cp.async.bulk.global.shared::cta.bulk_group [%0], [%1], %2;" ::"l"(gdst), "r"(smem_u32(ssrc)),
+               "r"(bytes)
+               : "memory");
+  asm volatile("cp.async.bulk.commit_group;" ::: "memory");
+}
+
+template <int N>
+__device__ __forceinline__ void bulk_wait_read() {
+  asm volatile("cp.async.bulk.wait_group.read %0;" ::"n"(N) : "memory");
+}
+
+__device__ __forceinline__ void bulk_wait_all() { asm volatile("cp.async.bulk.wait_group 0;" ::: "memory"); }
+
+template <bool SP, bool DP>
+__global__ void __launch_bounds__(32) copy_bulk(const CopyArgs a) {
+  extern __shared__ __align__(128) char smem[];
+  __shared__ __align__(8) uint64_t bar[kBulkStages];
+  if (threadIdx.x != 0) return;
+  const uint64_t ppc = (a.chunk + kBulkPiece - 1) / kBulkPiece;
+  const uint64_t items = uint64_t(a.nl) * uint64_t(a.n) * ppc;
+  if (blockIdx.x >= items) return;
+  const uint64_t mine = (items - blockIdx.x + gridDim.x - 1) / gridDim.x;
+  for (int i = 0; i < kBulkStages; ++i) mbar_init(&bar[i], 1);
+  asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+
+  auto piece = [&](uint64_t k, const char*& s, char*& d, uint32_t& bytes) {
+    const uint64_t w = blockIdx.x + k * gridDim.x;
+    const uint64_t c = w / ppc;
+    const uint64_t off = (w - c * ppc) * kBulkPiece;
+    item_ptrs<SP, DP>(a, c, s, d);
+    s += off;
+    d += off;
+    const uint64_t rem = a.chunk - off;
+    bytes = rem < kBulkPiece ? uint32_t(rem) : kBulkPiece;
+  };
+  const char* s;
+  char* d;
+  uint32_t nb;
+  for (uint64_t k = 0; k < mine && k < uint64_t(kBulkStages); ++k) {
+    piece(k, s, d, nb);
+    bulk_load(smem + k * kBulkPiece, s, nb, &bar[k]);
+  }
+  for (uint64_t k = 0; k < mine; ++k) {
+    const int st = int(k % kBulkStages);
+    mbar_wait(&bar[st], uint32_t((k / kBulkStages) & 1));
+    piece(k, s, d, nb);
+    bulk_store(d, smem + uint64_t(st) * kBulkPiece, nb);
+    if (k >= 1 && k - 1 + kBulkStages < mine) {
+      bulk_wait_read<1>();  // the store of item k-1 has finished reading its stage
+      const uint64_t kn = k - 1 + kBulkStages;
+      const int sn = int((k - 1) % kBulkStages);
+      piece(kn, s, d, nb);
+      bulk_load(smem + uint64_t(sn) * kBulkPiece, s, nb, &bar[sn]);
+    }
+  }
+  bulk_wait_all();
+}
+
+template <bool SP, bool DP>
+cudaError_t launch_t(const CopyArgs& a, int impl, int max_ctas, cudaStream_t s) {
+  const uint64_t items_lsu = uint64_t(a.nl) * a.n * ((a.chunk + kLsuPiece - 1) / kLsuPiece);
+  if (items_lsu == 0) return cudaSuccess;
+  if (impl == IMPL_BULK) {
+    static bool attr = false;
+    if (!attr) {
+      cudaError_t e = cudaFuncSetAttribute(copy_bulk<SP, DP>, cudaFuncAttributeMaxDynamicSharedMemorySize, kBulkSmem);
+      if (e != cudaSuccess) return e;
+      attr = true;
+    }
+    const uint64_t items = uint64_t(a.nl) * a.n * ((a.chunk + kBulkPiece - 1) / kBulkPiece);
+    uint64_t grid = max_ctas > 0 ? uint64_t(max_ctas) : uint64_t(kSMs);
+    if (grid > items) grid = items;
+    copy_bulk<SP, DP><<<unsigned(grid), 32, kBulkSmem, s>>>(a);
+  } else {
+    uint64_t grid = max_ctas > 0 ? uint64_t(max_ctas) : uint64_t(kSMs) * 4;
+    if (grid > items_lsu) grid = items_lsu;
+    copy_lsu<SP, DP><<<unsigned(grid), kLsuThreads, 0, s>>>(a);
+  }
+  return cudaGetLastError();
+}
+
+}  // namespace
+
+cudaError_t launch_copy(const CopyArgs& a, int impl, int max_ctas, cudaStream_t s) {
+  const bool sp = a.src_off != nullptr, dp = a.dst_off != nullptr;
+  if (sp && dp) return launch_t<true, true>(a, impl, max_ctas, s);
+  if (sp) return launch_t<true, false>(a, impl, max_ctas, s);
+  if (dp) return launch_t<false, true>(a, impl, max_ctas, s);
+  return launch_t<false, false>(a, impl, max_ctas, s);
+}
+
+// memmove semantics (reading 21): when the ranges overlap, copy in chunks of at most |dst - src|
+// bytes, ascending when dst < src and descending when dst > src, each chunk one launch on the
+// same stream so a chunk never reads bytes an earlier chunk overwrote.
+cudaError_t launch_memmove(char* base, uint64_t src_off, uint64_t dst_off, uint64_t bytes, int impl,
+                           cudaStream_t s, int* launches) {
+  *launches = 0;
+  if (bytes == 0 || src_off == dst_off) return cudaSuccess;
+  const uint64_t gap = src_off > dst_off ? src_off - dst_off : dst_off - src_off;
+  const uint64_t step = gap >= bytes ? bytes : gap;
+  const uint64_t nchunks = (bytes + step - 1) / step;
+  for (uint64_t q = 0; q < nchunks; ++q) {
+    const uint64_t k = dst_off < src_off ? q : nchunks - 1 - q;
+    const uint64_t off = k * step;
+    const uint64_t len = (bytes - off) < step ? (bytes - off) : step;
+    CopyArgs a;
+    a.src = base + src_off + off;
+    a.dst = base + dst_off + off;
+    a.chunk = len;
+    a.nl = 1;
+    a.n = 1;
+    cudaError_t e = launch_copy(a, impl, 0, s);
+    if (e != cudaSuccess) return e;
+    ++*launches;
+  }
+  return cudaSuccess;
+}
+
+}  // namespace aeg

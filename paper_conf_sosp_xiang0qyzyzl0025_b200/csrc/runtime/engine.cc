@@ -1,0 +1,441 @@
+// Context lifetime, transfers/events (rule ❶ readiness), the reclaim daemon (step ⑧), the block-
+// table arena, kernel timing and the primitive trace.
+#include "engine.h"
+
+#include <algorithm>
+#include <chrono>
+#include <cinttypes>
+#include <cstring>
+
+namespace aeg {
+
+namespace {
+constexpr uint64_t kMiB = 1ull << 20, kGiB = 1ull << 30;
+constexpr uint64_t kAlign = 2 * kMiB;
+}  // namespace
+
+// ------------------------------------------------------------------------------------ init
+void Ctx::init(int dev, const aeg_config& c) {
+  cfg = c;
+  host_only = (cfg.flags & AEG_CFG_HOST_ONLY) != 0;
+  timing = (cfg.flags & AEG_CFG_TIMING) != 0;
+  AEG_REQUIRE(cfg.dev_slab_bytes > 0 && cfg.host_slab_bytes > 0, AEG_ERR_INVALID, "slab sizes must be > 0");
+  pool[AEG_POOL_DEVICE].init(AEG_POOL_DEVICE, cfg.device_kv_bytes, cfg.dev_slab_bytes, cfg.dev_slab_layout);
+  pool[AEG_POOL_HOST].init(AEG_POOL_HOST, cfg.host_kv_bytes, cfg.host_slab_bytes, cfg.host_slab_layout);
+  for (auto& p : pool) p.is_done = [this](uint64_t x) { return is_done(x); };
+  if (host_only) {
+    if (!(cfg.flags & AEG_CFG_NO_DAEMON)) daemon = std::thread([this] { daemon_loop(); });
+    return;
+  }
+  device = dev;
+  CUDA_TRY(cudaSetDevice(device));
+  CUDA_TRY(cudaFree(nullptr));  // create / retain the primary context
+  AEG_REQUIRE(cfg.staging_slots >= 2, AEG_ERR_INVALID, "need at least 2 staging slots");
+  AEG_REQUIRE(cfg.staging_slot_bytes >= 1 * kMiB && cfg.staging_slot_bytes % 256 == 0, AEG_ERR_INVALID,
+              "staging slot must be >= 1 MiB and 256-byte aligned");
+  AEG_REQUIRE(cfg.stage_chunk_bytes >= 1 * kMiB && cfg.stage_ring_bytes >= 2 * cfg.stage_chunk_bytes,
+              AEG_ERR_INVALID, "stage ring must hold >= 2 chunks of >= 1 MiB");
+
+  // One device allocation: [KV | weights | out ring | in ring | tables]
+  const uint64_t kv = align_up(cfg.device_kv_bytes, kAlign);
+  const uint64_t w = align_up(cfg.device_weight_bytes, kAlign);
+  const uint64_t ring = align_up(cfg.staging_slot_bytes * cfg.staging_slots, kAlign);
+  const uint64_t tab = align_up(cfg.table_arena_bytes, kAlign);
+  dev_mem_bytes = kv + w + 2 * ring + tab;
+  CUDA_TRY(cudaMalloc(&dev_mem, dev_mem_bytes));
+  dev_kv = dev_mem;
+  dev_w = dev_mem + kv;
+  ring_out.base = dev_mem + kv + w;
+  ring_in.base = ring_out.base + ring;
+  tables.dev = ring_in.base + ring;
+  tables.bytes = tab;
+
+  // One pinned host allocation, pinned once: [CPU KV | Stage Buffer | tables]
+  const uint64_t hkv = align_up(cfg.host_kv_bytes, kAlign);
+  const uint64_t hst = align_up(cfg.stage_ring_bytes, kAlign);
+  host_mem_bytes = hkv + hst + tab;
+  CUDA_TRY(cudaHostAlloc(reinterpret_cast<void**>(&host_mem), host_mem_bytes,
+                         cudaHostAllocPortable | cudaHostAllocMapped));
+  host_kv = host_mem;
+  host_stage = host_mem + hkv;
+  tables.host = host_stage + hst;
+
+  int lo = 0, hi = 0;
+  CUDA_TRY(cudaDeviceGetStreamPriorityRange(&lo, &hi));
+  // copy-engine streams and the kernel streams; the gather/scatter/migrate kernels get the highest
+  // priority so they never queue behind long decode kernels of the caller.
+  CUDA_TRY(cudaStreamCreateWithPriority(&s_gather, cudaStreamNonBlocking, hi));
+  CUDA_TRY(cudaStreamCreateWithPriority(&s_scatter, cudaStreamNonBlocking, hi));
+  CUDA_TRY(cudaStreamCreateWithPriority(&s_migrate, cudaStreamNonBlocking, hi));
+  CUDA_TRY(cudaStreamCreateWithFlags(&s_d2h, cudaStreamNonBlocking));
+  CUDA_TRY(cudaStreamCreateWithFlags(&s_h2d, cudaStreamNonBlocking));
+  CUDA_TRY(cudaStreamCreateWithFlags(&s_weights, cudaStreamNonBlocking));
+  CUDA_TRY(cudaEventCreateWithFlags(&fence_ev, cudaEventDisableTiming));
+  for (Ring* r : {&ring_out, &ring_in}) {
+    r->slot_bytes = cfg.staging_slot_bytes;
+    r->n = cfg.staging_slots;
+    r->full.resize(r->n);
+    r->free_.resize(r->n);
+    for (int i = 0; i < r->n; ++i) {
+      CUDA_TRY(cudaEventCreateWithFlags(&r->full[i], cudaEventDisableTiming));
+      CUDA_TRY(cudaEventCreateWithFlags(&r->free_[i], cudaEventDisableTiming));
+    }
+  }
+  weights_start();
+  if (!(cfg.flags & AEG_CFG_NO_DAEMON)) daemon = std::thread([this] { daemon_loop(); });
+}
+
+void Ctx::shutdown() {
+  if (!host_only) {
+    weights_stop();
+    cudaSetDevice(device);
+    for (cudaStream_t s : {s_gather, s_d2h, s_h2d, s_scatter, s_weights, s_migrate})
+      if (s) cudaStreamSynchronize(s);
+  }
+  {
+    std::lock_guard<std::mutex> g(mu);
+    stop = true;
+  }
+  cv.notify_all();
+  if (daemon.joinable()) daemon.join();
+  if (host_only) return;
+  for (auto& kv : xfers) {
+    Xfer* x = kv.second.get();
+    if (!x->owns_events) continue;
+    for (cudaEvent_t e : x->ev) cudaEventDestroy(e);
+    if (x->done_ev) cudaEventDestroy(x->done_ev);
+  }
+  xfers.clear();
+  for (cudaEvent_t e : ev_pool) cudaEventDestroy(e);
+  for (cudaEvent_t e : ev_pool_ipc) cudaEventDestroy(e);
+  for (cudaEvent_t e : timing_pool) cudaEventDestroy(e);
+  for (auto& t : pending_timing) {
+    cudaEventDestroy(t.a);
+    cudaEventDestroy(t.b);
+  }
+  for (Ring* r : {&ring_out, &ring_in}) {
+    for (cudaEvent_t e : r->full) cudaEventDestroy(e);
+    for (cudaEvent_t e : r->free_) cudaEventDestroy(e);
+  }
+  for (auto& kv : peers) {
+    Peer* p = kv.second.get();
+    for (auto& e : p->events) cudaEventDestroy(e.second);
+    if (p->ipc_base) cudaIpcCloseMemHandle(p->ipc_base);
+  }
+  for (auto& r : registered) cudaHostUnregister(r.first);
+  cudaEventDestroy(fence_ev);
+  for (cudaStream_t s : {s_gather, s_d2h, s_h2d, s_scatter, s_weights, s_migrate})
+    if (s) cudaStreamDestroy(s);
+  if (dev_mem) cudaFree(dev_mem);
+  if (host_mem) cudaFreeHost(host_mem);
+}
+
+// ------------------------------------------------------------------------------- daemon ⑧
+void Ctx::daemon_loop() {
+  if (!host_only) cudaSetDevice(device);
+  std::unique_lock<std::mutex> lk(mu);
+  while (!stop) {
+    housekeeping();
+    cv.wait_for(lk, std::chrono::milliseconds(1));
+  }
+}
+
+bool Ctx::is_done(uint64_t x) {
+  auto it = xfers.find(x);
+  return it == xfers.end() || it->second->complete.load(std::memory_order_acquire);
+}
+
+void Ctx::poll() {
+  if (host_only) {
+    for (auto& kv : xfers)
+      if (kv.second->debug_done) kv.second->complete.store(true);
+    return;
+  }
+  for (auto& kv : xfers) {
+    Xfer* x = kv.second.get();
+    if (x->complete.load() || !x->done_recorded) continue;
+    cudaError_t e = cudaEventQuery(x->done_ev);
+    if (e == cudaSuccess) {
+      x->complete.store(true, std::memory_order_release);
+      if (tracing) {
+        char b[64];
+        snprintf(b, sizeof b, "sync %p", (void*)x->done_ev);
+        tr(b);
+      }
+    } else if (e != cudaErrorNotReady) {
+      (void)cudaGetLastError();
+    }
+  }
+}
+
+void Ctx::housekeeping() {
+  poll();
+  pool[0].reclaim();
+  pool[1].reclaim();
+  // release table-arena ranges of completed transfers (FIFO)
+  while (!tables.live.empty() && is_done(tables.live.front().xid)) tables.live.pop_front();
+  // reap released + completed transfers, recycle their events
+  for (auto it = xfers.begin(); it != xfers.end();) {
+    Xfer* x = it->second.get();
+    if (x->released && x->complete.load()) {
+      if (x->owns_events && !host_only) {
+        for (cudaEvent_t e : x->ev) give_event(e, x->ipc);
+        if (x->done_ev) give_event(x->done_ev, x->ipc);
+      }
+      it = xfers.erase(it);
+    } else {
+      ++it;
+    }
+  }
+  static int sweep = 0;
+  if (++sweep % 64 == 0) {
+    pool[0].forget_completed();
+    pool[1].forget_completed();
+  }
+  cv.notify_all();
+}
+
+// -------------------------------------------------------------------------------- events
+cudaEvent_t Ctx::take_event(bool ipc) {
+  auto& p = ipc ? ev_pool_ipc : ev_pool;
+  if (!p.empty()) {
+    cudaEvent_t e = p.back();
+    p.pop_back();
+    return e;
+  }
+  cudaEvent_t e;
+  CUDA_TRY(cudaEventCreateWithFlags(&e, ipc ? (cudaEventDisableTiming | cudaEventInterprocess) : cudaEventDisableTiming));
+  return e;
+}
+
+void Ctx::give_event(cudaEvent_t e, bool ipc) { (ipc ? ev_pool_ipc : ev_pool).push_back(e); }
+
+Xfer* Ctx::new_xfer(int kind, int32_t L, bool ipc) {
+  auto x = std::make_unique<Xfer>();
+  x->id = next_xid++;
+  x->kind = kind;
+  x->L = L;
+  x->ipc = ipc;
+  x->recorded.assign(L, 0);
+  if (!host_only) {
+    x->ev.resize(L);
+    for (int32_t l = 0; l < L; ++l) x->ev[l] = take_event(ipc);
+    x->done_ev = take_event(ipc);
+  }
+  Xfer* raw = x.get();
+  xfers.emplace(raw->id, std::move(x));
+  return raw;
+}
+
+Xfer* Ctx::get_xfer(uint64_t id) {
+  auto it = xfers.find(id);
+  AEG_REQUIRE(it != xfers.end() && !it->second->released, AEG_ERR_STATE, "unknown or released transfer %llu",
+              (unsigned long long)id);
+  return it->second.get();
+}
+
+void Ctx::record(Xfer* x, int32_t layer, cudaStream_t s) {
+  cudaEvent_t e = layer < 0 ? x->done_ev : x->ev[layer];
+  CUDA_TRY(cudaEventRecord(e, s));
+  tr_record(s, e);
+  if (layer < 0)
+    x->done_recorded = true;
+  else
+    x->recorded[layer] = 1;
+}
+
+// Rule ❷/❸: make stream s wait for the per-layer events [la, lb) of the incomplete transfers in
+// deps (per-layer granularity, reading 12; transfers without matching layers: their done event).
+void Ctx::wait_deps(cudaStream_t s, const std::vector<uint64_t>& deps, int32_t la, int32_t lb) {
+  for (uint64_t d : deps) {
+    auto it = xfers.find(d);
+    if (it == xfers.end() || it->second->complete.load()) continue;
+    Xfer* x = it->second.get();
+    for (int32_t l = la; l < lb; ++l) {
+      cudaEvent_t e;
+      if (x->kind != X_WEIGHTS && x->kind != X_RELOCATE && x->L > l && x->recorded[l])
+        e = x->ev[l];
+      else if (x->done_recorded)
+        e = x->done_ev;
+      else
+        fail(AEG_ERR_STATE, "dependency transfer %llu has unrecorded events", (unsigned long long)d);
+      CUDA_TRY(cudaStreamWaitEvent(s, e, 0));
+      tr_wait(s, e);
+    }
+  }
+}
+
+// Rule ❶ (Table 2).
+int Ctx::layer_ready(uint64_t id, int32_t layer, int mode, cudaStream_t s) {
+  std::unique_lock<std::mutex> lk(mu);
+  Xfer* x = get_xfer(id);
+  AEG_REQUIRE(layer >= -1 && layer < x->L, AEG_ERR_INVALID, "layer %d out of range [-1, %d)", layer, x->L);
+  AEG_REQUIRE(mode >= AEG_READY_QUERY && mode <= AEG_READY_BLOCK, AEG_ERR_INVALID, "bad mode %d", mode);
+  if (host_only) {
+    AEG_REQUIRE(mode == AEG_READY_QUERY, AEG_ERR_STATE, "host-only context: QUERY only");
+    return x->complete.load() ? AEG_OK : AEG_NOT_READY;
+  }
+  auto recorded = [&] { return layer < 0 ? x->done_recorded : x->recorded[layer] != 0; };
+  if (!recorded()) {
+    if (mode == AEG_READY_QUERY) return AEG_NOT_READY;
+    // weights pipeline: the event is recorded when its chunk is issued; wait for that on the host
+    cv.wait(lk, [&] { return recorded() || stop; });
+    AEG_REQUIRE(recorded(), AEG_ERR_STATE, "context shut down");
+  }
+  cudaEvent_t e = layer < 0 ? x->done_ev : x->ev[layer];
+  if (mode == AEG_READY_QUERY) {
+    if (x->complete.load()) return AEG_OK;
+    cudaError_t r = cudaEventQuery(e);
+    if (r == cudaSuccess) return AEG_OK;
+    if (r == cudaErrorNotReady) return AEG_NOT_READY;
+    fail(AEG_ERR_CUDA, "cudaEventQuery: %s", cudaGetErrorString(r));
+  }
+  if (mode == AEG_READY_WAIT_STREAM) {
+    CUDA_TRY(cudaStreamWaitEvent(s, e, 0));
+    tr_wait(s, e);
+    return AEG_OK;
+  }
+  lk.unlock();  // BLOCK: the transfer stays alive until released by this caller
+  CUDA_TRY(cudaEventSynchronize(e));
+  lk.lock();
+  if (tracing) {
+    char b[64];
+    snprintf(b, sizeof b, "sync %p", (void*)e);
+    tr(b);
+  }
+  return AEG_OK;
+}
+
+// --------------------------------------------------------------------------- table arena
+// FIFO ring: live entries are [oldest.start, head) circularly.  A request that does not fit
+// waits for the oldest transfers to complete.
+uint64_t Ctx::alloc_table(uint64_t bytes, uint64_t xid, char** host, char** dev) {
+  bytes = align_up(bytes, 256);
+  AEG_REQUIRE(bytes <= tables.bytes / 2, AEG_ERR_INVALID, "block table of %llu bytes exceeds the arena",
+              (unsigned long long)bytes);
+  for (;;) {
+    bool ok = false;
+    uint64_t start = 0;
+    if (tables.live.empty()) {
+      tables.head = 0;
+      ok = true;
+    } else {
+      const uint64_t oldest = tables.live.front().start;
+      if (tables.head > oldest) {
+        if (tables.head + bytes <= tables.bytes) {
+          start = tables.head;
+          ok = true;
+        } else if (bytes <= oldest) {
+          start = 0;
+          ok = true;
+        }
+      } else if (tables.head + bytes <= oldest) {
+        start = tables.head;
+        ok = true;
+      }
+    }
+    if (ok) {
+      if (tables.live.empty()) start = 0;
+      tables.head = start + bytes;
+      tables.live.push_back({xid, start, tables.head});
+      *host = tables.host + start;
+      *dev = tables.dev + start;
+      return start;
+    }
+    uint64_t oldest = tables.live.front().xid;
+    auto it = xfers.find(oldest);
+    if (it != xfers.end() && it->second->done_recorded) CUDA_TRY(cudaEventSynchronize(it->second->done_ev));
+    housekeeping();
+  }
+}
+
+// ----------------------------------------------------------------------- kernels + timing
+void Ctx::launch(int kind, const CopyArgs& a, cudaStream_t s, int impl, int max_ctas) {
+  cudaEvent_t ta = nullptr, tb = nullptr;
+  if (timing) {
+    auto take = [&]() {
+      if (!timing_pool.empty()) {
+        cudaEvent_t e = timing_pool.back();
+        timing_pool.pop_back();
+        return e;
+      }
+      cudaEvent_t e;
+      CUDA_TRY(cudaEventCreate(&e));
+      return e;
+    };
+    ta = take();
+    tb = take();
+    CUDA_TRY(cudaEventRecord(ta, s));
+  }
+  cudaError_t e = launch_copy(a, impl, max_ctas, s);
+  AEG_REQUIRE(e == cudaSuccess, AEG_ERR_CUDA, "copy kernel launch failed: %s", cudaGetErrorString(e));
+  kstats[kind].launches++;
+  kstats[kind].bytes += 2 * a.chunk * uint64_t(a.nl) * uint64_t(a.n);
+  if (timing) {
+    CUDA_TRY(cudaEventRecord(tb, s));
+    pending_timing.push_back({kind, ta, tb});
+    if (pending_timing.size() > 4096) resolve_timing(true);
+  }
+}
+
+void Ctx::resolve_timing(bool block) {
+  std::vector<TimingRec> keep;
+  for (auto& t : pending_timing) {
+    if (block) cudaEventSynchronize(t.b);
+    float ms = 0;
+    cudaError_t e = cudaEventElapsedTime(&ms, t.a, t.b);
+    if (e == cudaSuccess) {
+      kstats[t.kind].ms += ms;
+      timing_pool.push_back(t.a);
+      timing_pool.push_back(t.b);
+    } else {
+      (void)cudaGetLastError();
+      keep.push_back(t);
+    }
+  }
+  pending_timing.swap(keep);
+}
+
+// ---------------------------------------------------------------------------------- trace
+std::string Ctx::sname(cudaStream_t s) const {
+  if (s == s_gather) return "gather";
+  if (s == s_d2h) return "d2h";
+  if (s == s_h2d) return "h2d";
+  if (s == s_scatter) return "scatter";
+  if (s == s_weights) return "weights";
+  if (s == s_migrate) return "migrate";
+  char b[32];
+  snprintf(b, sizeof b, "u%p", (void*)s);
+  return b;
+}
+
+void Ctx::tr_record(cudaStream_t s, cudaEvent_t e) {
+  if (!tracing) return;
+  char b[96];
+  snprintf(b, sizeof b, "record %s %p", sname(s).c_str(), (void*)e);
+  tr(b);
+}
+
+void Ctx::tr_wait(cudaStream_t s, cudaEvent_t e) {
+  if (!tracing) return;
+  char b[96];
+  snprintf(b, sizeof b, "wait %s %p", sname(s).c_str(), (void*)e);
+  tr(b);
+}
+
+std::string Ctx::cells(int tag, const SlabPool& p, const aeg_block* b, int32_t n, int32_t la, int32_t lb,
+                       int32_t i0, int32_t i1) const {
+  (void)p;
+  (void)n;
+  std::string out;
+  char buf[64];
+  const char* t = tag == 0 ? "D" : tag == 1 ? "H" : "P";
+  for (int32_t l = la; l < lb; ++l)
+    for (int32_t i = i0; i < i1; ++i) {
+      snprintf(buf, sizeof buf, "%s%s:%u:%u:%d", out.empty() ? "" : ",", t, block_slab(b[i]), block_idx(b[i]), l);
+      out += buf;
+    }
+  return out;
+}
+
+}  // namespace aeg

@@ -1,0 +1,346 @@
+// KV movement (H2-H6): swap-out (gather kernel -> copy-engine D2H), swap-in (copy-engine H2D ->
+// scatter kernel), NVLink migrate (fused gather -> remote store) and weight relocation (N1).
+//
+// Every transfer is enqueued entirely from the calling thread, so all its events are recorded
+// before the call returns.  Stream roles (Fig. 10 "KV-Out" / "KV-In" streams):
+//   swap-out : s_gather (kernel, high priority)  ->  s_d2h     (copy engine)
+//   swap-in  : s_h2d    (copy engine)            ->  s_scatter (kernel, high priority)
+// The two halves of a direction hand staging slots back and forth with full/free events.
+#include <algorithm>
+#include <cstring>
+
+#include "engine.h"
+
+namespace aeg {
+
+namespace {
+
+constexpr uint64_t kPackLayerBytes = 4ull << 20;  // layers smaller than this share a segment
+
+struct Seg {
+  int32_t la, lb, i0, i1;
+};
+
+// A transfer of n blocks x L layers is cut into segments that fit one staging slot: whole layers
+// (several when a layer is tiny) or, for big layers, runs of blocks of one layer.  Segments are in
+// layer order, so the per-layer event can be recorded right after a layer's last segment.
+std::vector<Seg> plan(int32_t L, int32_t n, uint64_t chunk, uint64_t slot_bytes) {
+  std::vector<Seg> out;
+  if (n == 0) return out;
+  const uint64_t layer = uint64_t(n) * chunk;
+  if (layer <= slot_bytes) {
+    int32_t lps = 1;
+    if (layer < kPackLayerBytes)
+      lps = int32_t(std::max<uint64_t>(1, std::min<uint64_t>(kPackLayerBytes, slot_bytes) / layer));
+    lps = std::min(lps, L);
+    for (int32_t la = 0; la < L; la += lps) out.push_back({la, std::min(L, la + lps), 0, n});
+  } else {
+    const int32_t bps = int32_t(slot_bytes / chunk);
+    for (int32_t l = 0; l < L; ++l)
+      for (int32_t i0 = 0; i0 < n; i0 += bps) out.push_back({l, l + 1, i0, std::min(n, i0 + bps)});
+  }
+  return out;
+}
+
+// Maximal runs of host handles that are consecutive blocks of one slab.
+struct Run {
+  int32_t i0, m;
+  aeg_block first;
+};
+std::vector<Run> runs_of(const aeg_block* h, int32_t n) {
+  std::vector<Run> r;
+  for (int32_t i = 0; i < n;) {
+    int32_t m = 1;
+    while (i + m < n && block_slab(h[i + m]) == block_slab(h[i]) && block_idx(h[i + m]) == block_idx(h[i]) + uint32_t(m))
+      ++m;
+    r.push_back({i, m, h[i]});
+    i += m;
+  }
+  return r;
+}
+
+std::vector<uint64_t> uniq(std::vector<uint64_t> v) {
+  std::sort(v.begin(), v.end());
+  v.erase(std::unique(v.begin(), v.end()), v.end());
+  return v;
+}
+
+}  // namespace
+
+// Copy-engine DMAs between a staging slot and the host blocks of segment g (layer-major staging
+// image inside the slot).  dir = cudaMemcpyDeviceToHost (swap-out) or HostToDevice (swap-in).
+static void host_dmas(Ctx& c, const Shape& sh, const std::vector<Run>& runs, const Seg& g, char* slot,
+                      cudaMemcpyKind dir, cudaStream_t s) {
+  const SlabPool& hp = c.pool[AEG_POOL_HOST];
+  const uint64_t Cl = sh.chunk(), hstride = hp.lstride(sh);
+  const int32_t nseg = g.i1 - g.i0, nl = g.lb - g.la;
+  for (const Run& r : runs) {
+    const int32_t a = std::max(r.i0, g.i0), b = std::min(r.i0 + r.m, g.i1);
+    if (a >= b) continue;
+    const aeg_block hb = make_block(AEG_POOL_HOST, block_slab(r.first), block_idx(r.first) + uint32_t(a - r.i0));
+    const int32_t m = b - a;
+    char* host0 = c.host_kv + hp.off0(hb, sh) + uint64_t(g.la) * hstride;
+    char* st0 = slot + uint64_t(a - g.i0) * Cl;
+    const uint64_t st_pitch = uint64_t(nseg) * Cl;  // next layer inside the slot
+    if (hp.layout == AEG_LAYER_MAJOR) {
+      // the run is contiguous within each layer: one 1-D copy, or one 2-D copy over the layers
+      const uint64_t w = uint64_t(m) * Cl;
+      if (nl == 1) {
+        if (dir == cudaMemcpyDeviceToHost)
+          CUDA_TRY(cudaMemcpyAsync(host0, st0, w, dir, s));
+        else
+          CUDA_TRY(cudaMemcpyAsync(st0, host0, w, dir, s));
+      } else if (dir == cudaMemcpyDeviceToHost) {
+        CUDA_TRY(cudaMemcpy2DAsync(host0, hstride, st0, st_pitch, w, nl, dir, s));
+      } else {
+        CUDA_TRY(cudaMemcpy2DAsync(st0, st_pitch, host0, hstride, w, nl, dir, s));
+      }
+    } else {
+      // block-major: within a layer consecutive blocks are L*Cl apart -> one 2-D copy per layer
+      for (int32_t t = 0; t < nl; ++t) {
+        char* h = host0 + uint64_t(t) * hstride;
+        char* st = st0 + uint64_t(t) * st_pitch;
+        if (dir == cudaMemcpyDeviceToHost)
+          CUDA_TRY(cudaMemcpy2DAsync(h, sh.block(), st, Cl, Cl, m, dir, s));
+        else
+          CUDA_TRY(cudaMemcpy2DAsync(st, Cl, h, sh.block(), Cl, m, dir, s));
+      }
+    }
+  }
+}
+
+static int impl_of(const aeg_config& cfg) { return cfg.kernel == AEG_KERNEL_BULK ? IMPL_BULK : IMPL_LSU; }
+
+// ----------------------------------------------------------------------------- swap-out H3
+uint64_t Ctx::swap_out(const Shape& sh, const aeg_block* dev, const aeg_block* host, int32_t n, uint32_t flags) {
+  AEG_REQUIRE(!host_only, AEG_ERR_STATE, "host-only context has no data path");
+  SlabPool &dp = pool[AEG_POOL_DEVICE], &hp = pool[AEG_POOL_HOST];
+  dp.check_owned(dev, n, &sh);
+  hp.check_owned(host, n, &sh);
+  AEG_REQUIRE(sh.chunk() <= ring_out.slot_bytes, AEG_ERR_INVALID, "chunk larger than a staging slot");
+  Xfer* x = new_xfer(X_SWAP_OUT, sh.L, false);
+  std::vector<uint64_t> rdeps, wdeps;
+  if (!(flags & AEG_NO_DEPS)) {
+    for (int32_t i = 0; i < n; ++i) dp.deps_for_read(dev[i], rdeps);
+    for (int32_t i = 0; i < n; ++i) hp.deps_for_write(host[i], wdeps);
+  }
+  rdeps = uniq(rdeps);
+  wdeps = uniq(wdeps);
+  char *htab = nullptr, *dtab = nullptr;
+  if (n > 0) {
+    alloc_table(uint64_t(n) * 8, x->id, &htab, &dtab);
+    uint64_t* t = reinterpret_cast<uint64_t*>(htab);
+    for (int32_t i = 0; i < n; ++i) t[i] = dp.off0(dev[i], sh);
+    CUDA_TRY(cudaMemcpyAsync(dtab, htab, uint64_t(n) * 8, cudaMemcpyHostToDevice, s_gather));
+  }
+  const auto segs = plan(sh.L, n, sh.chunk(), ring_out.slot_bytes);
+  const auto runs = runs_of(host, n);
+  const uint64_t dstride = dp.lstride(sh);
+  for (const Seg& g : segs) {
+    const int slot = int(ring_out.next++ % uint64_t(ring_out.n));
+    char* sp = ring_out.slot(slot);
+    if (g.i0 == 0) wait_deps(s_gather, rdeps, g.la, g.lb);  // rule ❷
+    CUDA_TRY(cudaStreamWaitEvent(s_gather, ring_out.free_[slot], 0));
+    tr_wait(s_gather, ring_out.free_[slot]);
+    CopyArgs a;
+    a.src = dev_kv;
+    a.src_off = reinterpret_cast<const uint64_t*>(dtab) + g.i0;
+    a.src_lstride = dstride;
+    a.l_first = g.la;
+    a.dst = sp;
+    a.chunk = sh.chunk();
+    a.nl = g.lb - g.la;
+    a.n = g.i1 - g.i0;
+    launch(0, a, s_gather, impl_of(cfg), 0);
+    if (tracing) tr("op gather gather r=" + cells(0, dp, dev, n, g.la, g.lb, g.i0, g.i1) + " w=SO" + std::to_string(slot));
+    CUDA_TRY(cudaEventRecord(ring_out.full[slot], s_gather));
+    tr_record(s_gather, ring_out.full[slot]);
+
+    CUDA_TRY(cudaStreamWaitEvent(s_d2h, ring_out.full[slot], 0));
+    tr_wait(s_d2h, ring_out.full[slot]);
+    if (g.i0 == 0) wait_deps(s_d2h, wdeps, g.la, g.lb);  // rule ❸
+    host_dmas(*this, sh, runs, g, sp, cudaMemcpyDeviceToHost, s_d2h);
+    if (tracing) tr("op d2h d2h r=SO" + std::to_string(slot) + " w=" + cells(1, hp, host, n, g.la, g.lb, g.i0, g.i1));
+    CUDA_TRY(cudaEventRecord(ring_out.free_[slot], s_d2h));
+    tr_record(s_d2h, ring_out.free_[slot]);
+    if (g.i1 == n)
+      for (int32_t l = g.la; l < g.lb; ++l) record(x, l, s_d2h);
+  }
+  if (n == 0)
+    for (int32_t l = 0; l < sh.L; ++l) record(x, l, s_d2h);
+  record(x, -1, s_d2h);
+  for (int32_t i = 0; i < n; ++i) dp.note_read(dev[i], x->id);
+  for (int32_t i = 0; i < n; ++i) hp.note_write(host[i], x->id);
+  if (flags & AEG_FREE_SRC) dp.free(dev, n);
+  return x->id;
+}
+
+// ------------------------------------------------------------------------------ swap-in H4
+uint64_t Ctx::swap_in(const Shape& sh, const aeg_block* host, const aeg_block* dev, int32_t n, uint32_t flags) {
+  AEG_REQUIRE(!host_only, AEG_ERR_STATE, "host-only context has no data path");
+  SlabPool &dp = pool[AEG_POOL_DEVICE], &hp = pool[AEG_POOL_HOST];
+  hp.check_owned(host, n, &sh);
+  dp.check_owned(dev, n, &sh);
+  AEG_REQUIRE(sh.chunk() <= ring_in.slot_bytes, AEG_ERR_INVALID, "chunk larger than a staging slot");
+  Xfer* x = new_xfer(X_SWAP_IN, sh.L, false);
+  std::vector<uint64_t> rdeps, wdeps;
+  if (!(flags & AEG_NO_DEPS)) {
+    for (int32_t i = 0; i < n; ++i) hp.deps_for_read(host[i], rdeps);
+    for (int32_t i = 0; i < n; ++i) dp.deps_for_write(dev[i], wdeps);
+  }
+  rdeps = uniq(rdeps);
+  wdeps = uniq(wdeps);
+  char *htab = nullptr, *dtab = nullptr;
+  if (n > 0) {
+    alloc_table(uint64_t(n) * 8, x->id, &htab, &dtab);
+    uint64_t* t = reinterpret_cast<uint64_t*>(htab);
+    for (int32_t i = 0; i < n; ++i) t[i] = dp.off0(dev[i], sh);
+    CUDA_TRY(cudaMemcpyAsync(dtab, htab, uint64_t(n) * 8, cudaMemcpyHostToDevice, s_scatter));
+  }
+  const auto segs = plan(sh.L, n, sh.chunk(), ring_in.slot_bytes);
+  const auto runs = runs_of(host, n);
+  const uint64_t dstride = dp.lstride(sh);
+  for (const Seg& g : segs) {
+    const int slot = int(ring_in.next++ % uint64_t(ring_in.n));
+    char* sp = ring_in.slot(slot);
+    if (g.i0 == 0) wait_deps(s_h2d, rdeps, g.la, g.lb);  // rule ❷ per layer (reading 12)
+    CUDA_TRY(cudaStreamWaitEvent(s_h2d, ring_in.free_[slot], 0));
+    tr_wait(s_h2d, ring_in.free_[slot]);
+    host_dmas(*this, sh, runs, g, sp, cudaMemcpyHostToDevice, s_h2d);
+    if (tracing) tr("op h2d h2d r=" + cells(1, hp, host, n, g.la, g.lb, g.i0, g.i1) + " w=SI" + std::to_string(slot));
+    CUDA_TRY(cudaEventRecord(ring_in.full[slot], s_h2d));
+    tr_record(s_h2d, ring_in.full[slot]);
+
+    CUDA_TRY(cudaStreamWaitEvent(s_scatter, ring_in.full[slot], 0));
+    tr_wait(s_scatter, ring_in.full[slot]);
+    if (g.i0 == 0) wait_deps(s_scatter, wdeps, g.la, g.lb);  // rule ❸
+    CopyArgs a;
+    a.src = sp;
+    a.dst = dev_kv;
+    a.dst_off = reinterpret_cast<const uint64_t*>(dtab) + g.i0;
+    a.dst_lstride = dstride;
+    a.l_first = g.la;
+    a.chunk = sh.chunk();
+    a.nl = g.lb - g.la;
+    a.n = g.i1 - g.i0;
+    launch(1, a, s_scatter, impl_of(cfg), 0);
+    if (tracing) tr("op scatter scatter r=SI" + std::to_string(slot) + " w=" + cells(0, dp, dev, n, g.la, g.lb, g.i0, g.i1));
+    CUDA_TRY(cudaEventRecord(ring_in.free_[slot], s_scatter));
+    tr_record(s_scatter, ring_in.free_[slot]);
+    if (g.i1 == n)
+      for (int32_t l = g.la; l < g.lb; ++l) record(x, l, s_scatter);
+  }
+  if (n == 0)
+    for (int32_t l = 0; l < sh.L; ++l) record(x, l, s_scatter);
+  record(x, -1, s_scatter);
+  for (int32_t i = 0; i < n; ++i) hp.note_read(host[i], x->id);
+  for (int32_t i = 0; i < n; ++i) dp.note_write(dev[i], x->id);
+  if (flags & AEG_FREE_SRC) hp.free(host, n);
+  return x->id;
+}
+
+// ------------------------------------------------------------------------------- migrate H5
+uint64_t Ctx::migrate(const Shape& sh, const aeg_block* src, int32_t peer, const aeg_block* dst, int32_t n,
+                      uint32_t flags) {
+  AEG_REQUIRE(!host_only, AEG_ERR_STATE, "host-only context has no data path");
+  SlabPool& dp = pool[AEG_POOL_DEVICE];
+  dp.check_owned(src, n, &sh);
+  const SlabPool* dg = &dp;
+  char* dbase = dev_kv;
+  Peer* P = nullptr;
+  if (peer < 0) {
+    dp.check_owned(dst, n, &sh);
+    std::vector<aeg_block> all(src, src + n);
+    all.insert(all.end(), dst, dst + n);
+    std::sort(all.begin(), all.end());
+    AEG_REQUIRE(std::adjacent_find(all.begin(), all.end()) == all.end(), AEG_ERR_INVALID,
+                "local migrate: source and destination blocks overlap");
+  } else {
+    auto it = peers.find(peer);
+    AEG_REQUIRE(it != peers.end() && it->second->valid, AEG_ERR_INVALID, "peer %d not imported", peer);
+    P = it->second.get();
+    P->geom.check_geometry(dst, n, sh);
+    dg = &P->geom;
+    dbase = P->dev_kv;
+  }
+  Xfer* x = new_xfer(X_MIGRATE, sh.L, peer >= 0 && !P->same_process);
+  std::vector<uint64_t> rdeps, wdeps;
+  if (!(flags & AEG_NO_DEPS)) {
+    for (int32_t i = 0; i < n; ++i) dp.deps_for_read(src[i], rdeps);
+    if (peer < 0)
+      for (int32_t i = 0; i < n; ++i) dp.deps_for_write(dst[i], wdeps);
+  }
+  rdeps = uniq(rdeps);
+  wdeps = uniq(wdeps);
+  for (uint64_t d : wdeps) rdeps.push_back(d);
+  rdeps = uniq(rdeps);
+  char *htab = nullptr, *dtab = nullptr;
+  if (n > 0) {
+    alloc_table(uint64_t(n) * 16, x->id, &htab, &dtab);
+    uint64_t* t = reinterpret_cast<uint64_t*>(htab);
+    for (int32_t i = 0; i < n; ++i) t[i] = dp.off0(src[i], sh);
+    for (int32_t i = 0; i < n; ++i) t[n + i] = dg->off0(dst[i], sh);
+    CUDA_TRY(cudaMemcpyAsync(dtab, htab, uint64_t(n) * 16, cudaMemcpyHostToDevice, s_migrate));
+  }
+  const uint64_t layer = uint64_t(n) * sh.chunk();
+  int32_t lps = 1;
+  if (n > 0 && layer < kPackLayerBytes) lps = int32_t(std::min<uint64_t>(sh.L, std::max<uint64_t>(1, kPackLayerBytes / layer)));
+  const int impl = impl_of(cfg);
+  for (int32_t la = 0; la < sh.L; la += lps) {
+    const int32_t lb = std::min(sh.L, la + lps);
+    if (n > 0) {
+      wait_deps(s_migrate, rdeps, la, lb);
+      CopyArgs a;
+      a.src = dev_kv;
+      a.src_off = reinterpret_cast<const uint64_t*>(dtab);
+      a.src_lstride = dp.lstride(sh);
+      a.dst = dbase;
+      a.dst_off = reinterpret_cast<const uint64_t*>(dtab) + n;
+      a.dst_lstride = dg->lstride(sh);
+      a.l_first = la;
+      a.chunk = sh.chunk();
+      a.nl = lb - la;
+      a.n = n;
+      launch(2, a, s_migrate, impl, cfg.migrate_ctas);
+      if (tracing)
+        tr("op migrate migrate r=" + cells(0, dp, src, n, la, lb, 0, n) + " w=" + cells(peer < 0 ? 0 : 2, *dg, dst, n, la, lb, 0, n));
+    }
+    for (int32_t l = la; l < lb; ++l) record(x, l, s_migrate);
+  }
+  record(x, -1, s_migrate);
+  for (int32_t i = 0; i < n; ++i) dp.note_read(src[i], x->id);
+  if (peer < 0)
+    for (int32_t i = 0; i < n; ++i) dp.note_write(dst[i], x->id);
+  if (flags & AEG_FREE_SRC) dp.free(src, n);
+  return x->id;
+}
+
+// ------------------------------------------------------------------------------ relocate N1
+uint64_t Ctx::relocate(uint64_t src_off, uint64_t dst_off, uint64_t bytes) {
+  AEG_REQUIRE(!host_only, AEG_ERR_STATE, "host-only context has no data path");
+  const uint64_t W = cfg.device_weight_bytes;
+  AEG_REQUIRE(src_off + bytes <= W && dst_off + bytes <= W, AEG_ERR_INVALID, "relocation outside the weights region");
+  AEG_REQUIRE(src_off % 16 == 0 && dst_off % 16 == 0 && bytes % 16 == 0, AEG_ERR_INVALID,
+              "relocation offsets and size must be multiples of 16");
+  Xfer* x = new_xfer(X_RELOCATE, 1, false);
+  int nl = 0;
+  cudaEvent_t ta = nullptr, tb = nullptr;
+  if (timing) {
+    CUDA_TRY(cudaEventCreate(&ta));
+    CUDA_TRY(cudaEventCreate(&tb));
+    CUDA_TRY(cudaEventRecord(ta, s_weights));
+  }
+  cudaError_t e = launch_memmove(dev_w, src_off, dst_off, bytes, impl_of(cfg), s_weights, &nl);
+  AEG_REQUIRE(e == cudaSuccess, AEG_ERR_CUDA, "relocate launch failed: %s", cudaGetErrorString(e));
+  if (timing) {
+    CUDA_TRY(cudaEventRecord(tb, s_weights));
+    pending_timing.push_back({3, ta, tb});
+  }
+  kstats[3].launches += nl;
+  kstats[3].bytes += 2 * bytes;
+  record(x, 0, s_weights);
+  record(x, -1, s_weights);
+  return x->id;
+}
+
+}  // namespace aeg

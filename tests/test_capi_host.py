@@ -1,0 +1,211 @@
+"""CPU tests of the C-ABI library: it loads, exports every symbol include/aeg.h declares, and its
+slab allocator (host-only context, no CUDA) takes the same decisions as the oracle (O2), call by
+call, over exhaustive short and random long operation sequences on both pools."""
+import itertools
+import random
+import subprocess
+
+import numpy as np
+import pytest
+
+import paper_conf_sosp_xiang0qyzyzl0025_b200 as aeg
+from oracle.shape import KVShape
+from oracle.slab import AllocError, SlabPool
+
+
+@pytest.fixture(scope="module", autouse=True)
+def built():
+    from paper_conf_sosp_xiang0qyzyzl0025_b200 import build
+    build.build()
+
+
+def test_library_exports_every_declared_symbol():
+    declared = aeg.declared_symbols()
+    assert len(declared) >= 30
+    out = subprocess.run(["nm", "-D", "--defined-only", aeg.LIB_PATH], capture_output=True, text=True).stdout
+    exported = {line.split()[-1] for line in out.splitlines() if line.strip()}
+    missing = [s for s in declared if s not in exported]
+    assert not missing, missing
+    L = aeg.lib()
+    for s in declared:
+        assert hasattr(L, s)
+    # the binding covers the whole ABI
+    assert set(declared) == set(aeg._SIGS) | {"aeg_last_error"}
+
+
+def test_no_torch_in_abi():
+    src = open(aeg.HEADER).read()
+    assert "torch" not in src.replace("torch.distributed", "")
+    assert "at::" not in src and "Tensor" not in src
+
+
+A = (2, 1, 2, 2, 8)      # chunk 64 B, block 128 B
+Bs = (3, 1, 2, 2, 8)     # block 192 B
+SLAB = 256
+
+
+def host_ctx(n_slabs=3, layout=aeg.LAYER_MAJOR, **kw):
+    cfg = aeg.default_config(device_kv_bytes=n_slabs * SLAB, host_kv_bytes=n_slabs * SLAB, dev_slab_bytes=SLAB,
+                             host_slab_bytes=SLAB, dev_slab_layout=layout, host_slab_layout=layout,
+                             flags=aeg.CFG_HOST_ONLY | aeg.CFG_NO_DAEMON, **kw)
+    return aeg.Context(0, cfg)
+
+
+class Pair:
+    """Runs the same operations on the oracle pool and on the library (both pools)."""
+
+    def __init__(self, n_slabs, pool):
+        self.o = SlabPool(n_slabs * SLAB, SLAB)
+        self.c = host_ctx(n_slabs)
+        self.pool = pool
+        self.live, self.order, self.xfers = {}, [], []
+        self.tag = 0
+
+    def alloc(self, shape, n):
+        o_err = c_err = None
+        try:
+            o = self.o.alloc(KVShape(*shape), n)
+        except AllocError as e:
+            o, o_err = None, e.code
+        try:
+            c = self.c.kv_alloc(self.pool, shape, n)
+        except aeg.AegError as e:
+            c, c_err = None, e.code
+        assert o_err == c_err
+        if o is not None:
+            dec = [aeg.decode_block(b) for b in c]
+            assert all(p == self.pool for p, _, _ in dec)
+            assert [(s, j) for _, s, j in dec] == list(o)
+            self.live[self.tag] = (o, c)
+            self.order.append(self.tag)
+        self.tag += 1
+
+    def free(self, k):
+        if not self.order:
+            return
+        t = self.order.pop(k)
+        o, c = self.live.pop(t)
+        self.o.free(o)
+        self.c.kv_free(self.pool, c)
+
+    def xfer(self, k):
+        if not self.order:
+            return
+        o, c = self.live[self.order[k]]
+        self.xfers.append((self.o.begin(o), self.c.debug_xfer_begin(self.pool, c)))
+
+    def complete(self):
+        if self.xfers:
+            xo, xc = self.xfers.pop(0)
+            self.o.complete(xo)
+            self.c.debug_xfer_complete(xc)
+
+    def reclaim(self):
+        self.o.reclaim()
+        self.c.reclaim()
+
+    def compare_stats(self):
+        per, free = self.o.stats()
+        s = self.c.stats(self.pool)
+        assert s.free_slabs == free
+        got = {}
+        for i in range(s.n_shapes):
+            p = s.per_shape[i]
+            sh = KVShape(p.shape.num_layers, p.shape.num_kv_heads, p.shape.head_dim, p.shape.elem_bytes,
+                         p.shape.block_tokens)
+            got[sh] = (p.slabs, p.owned_blocks, p.quarantined_blocks)
+        assert got == per
+        used = sum(v[1] * sh.block_bytes() for sh, v in per.items())
+        assert s.used_bytes == used
+
+    def run(self, ops):
+        for op in ops:
+            getattr(self, op[0])(*op[1:])
+            self.compare_stats()
+
+
+OPS = [("alloc", A, 1), ("alloc", A, 2), ("alloc", A, 3), ("alloc", Bs, 1), ("alloc", Bs, 2),
+       ("free", 0), ("free", -1), ("xfer", 0), ("complete",), ("reclaim",)]
+
+
+@pytest.mark.parametrize("pool", [aeg.POOL_DEVICE, aeg.POOL_HOST])
+def test_allocator_matches_oracle_exhaustive(pool):
+    for seq in itertools.product(OPS, repeat=4):
+        p = Pair(3, pool)
+        p.run(seq)
+        p.c.shutdown()
+
+
+@pytest.mark.parametrize("seed", range(40))
+def test_allocator_matches_oracle_random(seed):
+    r = random.Random(seed)
+    p = Pair(5, seed % 2)
+    p.run([r.choice(OPS) for _ in range(120)])
+    p.c.shutdown()
+
+
+def test_error_codes_and_validation():
+    c = host_ctx(2)
+    b = c.kv_alloc(aeg.POOL_DEVICE, A, 2)
+    with pytest.raises(aeg.AegError) as e:
+        c.kv_free(aeg.POOL_HOST, b)                    # wrong pool
+    assert e.value.code == aeg.ERR_INVALID
+    with pytest.raises(aeg.AegError) as e:
+        c.kv_free(aeg.POOL_DEVICE, [b[0], b[0]])        # repeated
+    assert e.value.code == aeg.ERR_STATE
+    c.kv_free(aeg.POOL_DEVICE, b)
+    with pytest.raises(aeg.AegError) as e:
+        c.kv_free(aeg.POOL_DEVICE, b)                   # double free (slab reclaimed -> invalid)
+    assert e.value.code in (aeg.ERR_STATE, aeg.ERR_INVALID)
+    with pytest.raises(aeg.AegError) as e:
+        c.kv_alloc(aeg.POOL_DEVICE, (3, 2, 2, 2, 8), 1)  # block larger than a slab
+    assert e.value.code == aeg.ERR_INVALID
+    with pytest.raises(aeg.AegError) as e:
+        c.kv_alloc(aeg.POOL_DEVICE, A, 100)
+    assert e.value.code == aeg.ERR_OOM
+    with pytest.raises(aeg.AegError) as e:
+        c.kv_alloc(aeg.POOL_DEVICE, (0, 1, 2, 2, 8), 1)  # invalid shape
+    assert e.value.code == aeg.ERR_INVALID
+    with pytest.raises(aeg.AegError) as e:
+        c.kv_swap_out(A, [], [])                         # no data path in host-only mode
+    assert e.value.code == aeg.ERR_STATE
+    assert "host-only" in aeg.lib().aeg_last_error().decode()
+    assert len(c.kv_alloc(aeg.POOL_DEVICE, A, 0)) == 0
+    c.shutdown()
+
+
+def test_daemon_reclaims_move_list():
+    """With the daemon running, a move-list block is reclaimed without an explicit aeg_reclaim."""
+    import time
+    cfg = aeg.default_config(device_kv_bytes=2 * SLAB, host_kv_bytes=SLAB, dev_slab_bytes=SLAB,
+                             host_slab_bytes=SLAB, flags=aeg.CFG_HOST_ONLY)
+    c = aeg.Context(0, cfg)
+    b = c.kv_alloc(aeg.POOL_DEVICE, A, 2)
+    x = c.debug_xfer_begin(aeg.POOL_DEVICE, b)
+    c.kv_free(aeg.POOL_DEVICE, b)
+    assert c.stats(aeg.POOL_DEVICE).quarantined_blocks == 2
+    c.debug_xfer_complete(x)
+    for _ in range(200):
+        if c.stats(aeg.POOL_DEVICE).quarantined_blocks == 0:
+            break
+        time.sleep(0.005)
+    s = c.stats(aeg.POOL_DEVICE)
+    assert s.quarantined_blocks == 0 and s.free_slabs == 2
+    c.shutdown()
+
+
+def test_big_pool_alloc_is_fast():
+    """H1 control overhead: µs-scale per call even for thousands of blocks."""
+    import time
+    cfg = aeg.default_config(device_kv_bytes=160 << 30, host_kv_bytes=64 << 30, flags=aeg.CFG_HOST_ONLY | aeg.CFG_NO_DAEMON)
+    c = aeg.Context(0, cfg)
+    sh = (32, 32, 128, 2, 16)
+    t0 = time.perf_counter()
+    blocks = [c.kv_alloc(aeg.POOL_DEVICE, sh, 64) for _ in range(64)]
+    dt = time.perf_counter() - t0
+    assert dt < 0.5
+    for b in blocks[::2]:
+        c.kv_free(aeg.POOL_DEVICE, b)
+    got = c.kv_alloc(aeg.POOL_DEVICE, sh, 1024)
+    assert len(set(got.tolist())) == 1024
+    c.shutdown()
