@@ -202,6 +202,11 @@ int aegin_consume(const void* base, const uint64_t* dev_off, uint64_t n, uint64_
   return int(cudaGetLastError());
 }
 
+// Plain copy between any two pointers (device, pinned or pageable host) for test read-back.
+int aegin_copy(void* dst, const void* src, uint64_t n) { return int(cudaMemcpy(dst, src, n, cudaMemcpyDefault)); }
+
+int aegin_sync(void) { return int(cudaDeviceSynchronize()); }
+
 int aegin_spin(long long cycles, void* stream) {
   spin<<<1, 1, 0, static_cast<cudaStream_t>(stream)>>>(cycles);
   return int(cudaGetLastError());

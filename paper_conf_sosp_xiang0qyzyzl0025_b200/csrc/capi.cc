@@ -439,7 +439,10 @@ int aeg_import_peer(aeg_ctx ctx, int32_t peer, const void* buf, uint64_t len) {
     }
     p->valid = true;
     auto it = c.peers.find(peer);
-    if (it != c.peers.end() && it->second->ipc_base) cudaIpcCloseMemHandle(it->second->ipc_base);
+    if (it != c.peers.end()) {
+      if (it->second->ipc_base) cudaIpcCloseMemHandle(it->second->ipc_base);
+      p->events = std::move(it->second->events);
+    }
     c.peers[peer] = std::move(p);
     return AEG_OK;
   });
@@ -489,8 +492,10 @@ int aeg_xfer_import(aeg_ctx ctx, int32_t peer, const void* buf, uint64_t len, ae
     AEG_REQUIRE(same || h.ipc, AEG_ERR_INVALID, "transfer events are not interprocess-capable");
     std::lock_guard<std::mutex> g(c.mu);
     set_device(c);
+    AEG_REQUIRE(peer >= 0 && peer < 64, AEG_ERR_INVALID, "peer index out of range");
     auto it = c.peers.find(peer);
-    AEG_REQUIRE(it != c.peers.end(), AEG_ERR_INVALID, "peer %d not imported", peer);
+    if (it == c.peers.end())  // events only: the importer need not map the exporter's pool
+      it = c.peers.emplace(peer, std::make_unique<aeg::Peer>()).first;
     aeg::Peer* P = it->second.get();
     const cudaIpcEventHandle_t* hs =
         reinterpret_cast<const cudaIpcEventHandle_t*>(static_cast<const char*>(buf) + sizeof h);

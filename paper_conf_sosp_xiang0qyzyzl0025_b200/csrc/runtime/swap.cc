@@ -35,9 +35,12 @@ std::vector<Seg> plan(int32_t L, int32_t n, uint64_t chunk, uint64_t slot_bytes)
     lps = std::min(lps, L);
     for (int32_t la = 0; la < L; la += lps) out.push_back({la, std::min(L, la + lps), 0, n});
   } else {
-    const int32_t bps = int32_t(slot_bytes / chunk);
+    // balanced runs of blocks (no small tail segment): ceil(n / cap) segments of near-equal size
+    const int32_t cap = int32_t(slot_bytes / chunk);
+    const int32_t nseg = (n + cap - 1) / cap;
     for (int32_t l = 0; l < L; ++l)
-      for (int32_t i0 = 0; i0 < n; i0 += bps) out.push_back({l, l + 1, i0, std::min(n, i0 + bps)});
+      for (int32_t q = 0; q < nseg; ++q)
+        out.push_back({l, l + 1, int32_t(int64_t(n) * q / nseg), int32_t(int64_t(n) * (q + 1) / nseg)});
   }
   return out;
 }

@@ -123,9 +123,12 @@ struct WeightPipe {
   }
 
   void record_layers(WJob* j, const std::vector<uint64_t>& layer_last, uint64_t upto, cudaStream_t s) {
-    std::lock_guard<std::mutex> g(c->mu);
-    for (int32_t l = 0; l < j->x->L; ++l)
-      if (!j->x->recorded[l] && layer_last[l] != ~0ull && layer_last[l] < upto) c->record(j->x, l, s);
+    {
+      std::lock_guard<std::mutex> g(c->mu);
+      for (int32_t l = 0; l < j->x->L; ++l)
+        if (!j->x->recorded[l] && layer_last[l] != ~0ull && layer_last[l] < upto) c->record(j->x, l, s);
+    }
+    c->cv.notify_all();  // wake WAIT_STREAM / BLOCK readiness waiters (aeg_layer_ready)
   }
 
   void run_job(WJob* j) {

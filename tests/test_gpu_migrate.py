@@ -1,0 +1,144 @@
+"""GPU parity for H5 (prefill->decode KV hand-off): the fused migrate kernel's destination image
+equals oracle.kv.migrate (O7) — within one pool (peer -1), between two contexts of this process
+with different slab sizes/layouts (peer mapped directly), and between two processes through CUDA
+IPC memory and IPC events (the multi-process path of §8(e), exercised on one GPU)."""
+import multiprocessing as mp
+import os
+
+import numpy as np
+import pytest
+
+import aeg_inputs as gi
+import paper_conf_sosp_xiang0qyzyzl0025_b200 as aeg
+from oracle import kv as OK
+from oracle.shape import KVShape
+
+from .gpu_harness import Side, fill_blocks, first_diff, poison_blocks, require_gpu
+
+pytestmark = pytest.mark.gpu
+SH = KVShape(3, 2, 64, 2, 16)   # Cl = 8 KiB
+MIB = 1 << 20
+
+
+def make(layout, slab=MIB, nslabs=8, kernel=aeg.KERNEL_LSU):
+    cfg = aeg.default_config(device_kv_bytes=nslabs * slab, host_kv_bytes=MIB, dev_slab_bytes=slab,
+                             host_slab_bytes=MIB, dev_slab_layout=layout, staging_slot_bytes=MIB,
+                             staging_slots=2, stage_ring_bytes=4 * MIB, stage_chunk_bytes=MIB,
+                             table_arena_bytes=2 * MIB, host_threads=1, kernel=kernel)
+    ctx = aeg.Context(0, cfg)
+    return ctx, Side(ctx, aeg.POOL_DEVICE, cfg.device_kv_bytes, slab, layout)
+
+
+@pytest.mark.parametrize("kernel", [aeg.KERNEL_LSU, aeg.KERNEL_BULK])
+def test_local_migrate(kernel):
+    require_gpu()
+    ctx, dev = make(aeg.BLOCK_MAJOR, kernel=kernel)
+    try:
+        dev.poison(gi.TAG_NEVER)
+        img = dev.poison_img(gi.TAG_NEVER)
+        sc, so = dev.alloc(SH, 37)
+        fill_blocks(dev, img, SH, so, [(0, j) for j in range(37)])
+        dc, do = dev.alloc(SH, 37)
+        poison_blocks(dev, img, SH, do)
+        x = ctx.kv_migrate(SH.as_tuple(), sc, -1, dc)
+        exp = OK.migrate(img, dev.geom, img, dev.geom, SH, so, do)
+        ctx.layer_ready(x, -1, aeg.READY_BLOCK)
+        assert first_diff(dev.read(), exp) is None
+    finally:
+        ctx.shutdown()
+
+
+def test_same_process_peer_migrate_and_imported_events():
+    require_gpu()
+    a, A = make(aeg.LAYER_MAJOR, slab=MIB)
+    b, B = make(aeg.BLOCK_MAJOR, slab=MIB + 64 * 1024, nslabs=6)
+    try:
+        A.poison(gi.TAG_NEVER)
+        B.poison(gi.TAG_NEVER)
+        aimg, bimg = A.poison_img(gi.TAG_NEVER), B.poison_img(gi.TAG_NEVER)
+        sc, so = A.alloc(SH, 50)
+        fill_blocks(A, aimg, SH, so, [(3, j) for j in range(50)])
+        dc, do = B.alloc(SH, 50)
+        poison_blocks(B, bimg, SH, do)
+        a.import_peer(5, b.export_ipc())
+        b.import_peer(0, a.export_ipc())
+        x = a.kv_migrate(SH.as_tuple(), sc, 5, dc)
+        xi = b.xfer_import(0, a.xfer_export(x))
+        for l in range(SH.L):
+            b.layer_ready(xi, l, aeg.READY_BLOCK)
+        exp = OK.migrate(aimg, A.geom, bimg, B.geom, SH, so, do)
+        assert first_diff(B.read(), exp) is None
+        assert first_diff(A.read(), aimg) is None
+    finally:
+        a.shutdown()
+        b.shutdown()
+
+
+def _decode_side(conn):
+    """Child process: the decode instance.  Allocates destination blocks, exports its pool, waits on
+    the imported per-layer events, then reports its image."""
+    try:
+        _decode_body(conn)
+    except BaseException:
+        import traceback
+        conn.send(("error", traceback.format_exc()))
+        raise
+
+
+def _decode_body(conn):
+    ctx, dev = make(aeg.BLOCK_MAJOR, slab=MIB, nslabs=4)
+    dev.poison(gi.TAG_NEVER)
+    dc, do = dev.alloc(SH, 20)
+    img = dev.poison_img(gi.TAG_NEVER)
+    poison_blocks(dev, img, SH, do)
+    conn.send((ctx.export_ipc(), [int(b) for b in dc], do))
+    blob = conn.recv()
+    x = ctx.xfer_import(0, blob)
+    for l in range(SH.L):
+        ctx.layer_ready(x, l, aeg.READY_BLOCK)
+    conn.send(dev.read().tobytes())
+    conn.recv()
+    ctx.shutdown()
+
+
+def test_two_process_ipc_migrate():
+    require_gpu()
+    ctxm = mp.get_context("spawn")
+    parent, child = ctxm.Pipe()
+    p = ctxm.Process(target=_decode_side, args=(child,))
+    p.start()
+    child.close()
+
+    def recv():
+        assert parent.poll(120), "decode process did not answer"
+        m = parent.recv()
+        if isinstance(m, tuple) and len(m) == 2 and m[0] == "error":
+            raise AssertionError("decode process failed:\n" + m[1])
+        return m
+
+    try:
+        a, A = make(aeg.LAYER_MAJOR, slab=MIB, nslabs=4)
+        A.poison(gi.TAG_NEVER)
+        aimg = A.poison_img(gi.TAG_NEVER)
+        sc, so = A.alloc(SH, 20)
+        fill_blocks(A, aimg, SH, so, [(7, j) for j in range(20)])
+        blob, dc, do = recv()
+        a.import_peer(0, blob)
+        x = a.kv_migrate(SH.as_tuple(), sc, 0, np.array(dc, dtype=np.uint64), flags=aeg.FREE_SRC)
+        parent.send(a.xfer_export(x))
+        got = np.frombuffer(recv(), dtype=np.uint8)
+        geom = OK.PoolGeom(4 * MIB, MIB, aeg.BLOCK_MAJOR)
+        bimg = gi.region_bytes(gi.kv_seed(1), gi.poison_key(gi.TAG_NEVER, 0), geom.nbytes)
+        for h in do:
+            for l in range(SH.L):
+                o = OK.addr(geom, SH, h, l)
+                bimg[o:o + SH.chunk_bytes()] = gi.region_bytes(gi.kv_seed(1), gi.poison_key(gi.TAG_DST, o), SH.chunk_bytes())
+        exp = OK.migrate(aimg, A.geom, bimg, geom, SH, so, do)
+        assert first_diff(got, exp) is None
+        parent.send("bye")
+        a.shutdown()
+    finally:
+        p.join(timeout=30)
+        if p.is_alive():
+            p.kill()
+    assert p.exitcode == 0
