@@ -62,6 +62,8 @@ def parse():
     p.add_argument("--no-e2e", action="store_true")
     p.add_argument("--no-cpu", action="store_true")
     p.add_argument("--switches", type=int, default=30)
+    p.add_argument("--slot-mib", type=int, default=0, help="staging slot size (0 = library default)")
+    p.add_argument("--slots", type=int, default=0)
     p.add_argument("--profile", action="store_true", help="short run for ncu (no side legs)")
     return p.parse_args()
 
@@ -191,7 +193,7 @@ def c2_requests(n_req: int):
 class SwapBench:
     """configs[1] on one GPU: aged device pool, a 64-request batch, swap round trips."""
 
-    def __init__(self, aeg, sh, n_req, kernel, extra_host_slabs=8, weight_bytes=0, seed_cfg=2):
+    def __init__(self, aeg, sh, n_req, kernel, extra_host_slabs=8, weight_bytes=0, seed_cfg=2, slot_mib=0, slots=0):
         import aeg_inputs as gi
         from oracle import kv as OK
         from oracle.shape import KVShape
@@ -211,6 +213,11 @@ class SwapBench:
         self.seed = gi.kv_seed(seed_cfg)
         cfg = aeg.default_config(device_kv_bytes=dev_slabs * GIB, host_kv_bytes=host_slabs * GIB,
                                  device_weight_bytes=weight_bytes, kernel=kernel, flags=aeg.CFG_TIMING)
+        if slot_mib:
+            cfg.staging_slot_bytes = slot_mib * MIB
+        if slots:
+            cfg.staging_slots = slots
+        self.cfg = cfg
         t0 = time.time()
         self.ctx = aeg.Context(0, cfg)
         self.init_s = time.time() - t0
@@ -408,17 +415,11 @@ def pcie_calibration(torch):
     return out
 
 
-def switch_leg(aeg, torch, n_switch, kernel):
-    """configs[3]: token-level switch among Qwen-1.8B / Llama-7B / Yi-9B shapes on one GPU.
-    switch(A->B) = swap-out of A's 1 GiB decode KV (D2H) || staging of B's weights (H2D, PAPER.md
-    §5.2) -> swap-in of B's 1 GiB KV (H2D) -> per-layer consumer (weights layer i+1 and KV layer i).
-    Latency is from the switch start to the last (and first) layer ready, on the device timeline."""
+def model_caches(names):
+    """Host Model Caches (pageable) with generated bf16 content."""
     import aeg_inputs as gi
     from aeg_inputs import dev as D
-    names = ["qwen-1.8b", "llama-7b", "yi-9b"]
-    shapes = {n: gi.KV_SHAPES[n] for n in names}
     descs, caches = {}, {}
-    t0 = time.time()
     for m, nm in enumerate(names):
         ts = gi.model_tensors(nm)
         sizes = [t["rows"] * t["cols"] * 2 for t in ts]
@@ -429,49 +430,75 @@ def switch_leg(aeg, torch, n_switch, kernel):
         caches[nm] = buf
         descs[nm] = [dict(host_src=buf.ctypes.data + int(o), rows=t["rows"], cols=t["cols"], elem_bytes=2,
                           layer=t["layer"], split=t["split"], groups=t["groups"]) for t, o in zip(ts, offs)]
-    gen_s = time.time() - t0
-    wmax = max(int(c.nbytes) for c in caches.values()) + 64 * MIB
-    cfg = aeg.default_config(device_kv_bytes=8 * GIB, host_kv_bytes=8 * GIB, device_weight_bytes=wmax,
+    return descs, caches
+
+
+def switch_leg(aeg, torch, n_switch, kernel, descs, mode="staged"):
+    """configs[3]: token-level switch among Qwen-1.8B / Llama-7B / Yi-9B shapes on one GPU.
+    staged  : switch(A->B) = swap-out of A's 1 GiB decode KV (D2H) || staging of B's weights through
+              the pinned Stage Buffer (H2D, Fig. 9 3.a) -> swap-in of B's KV.
+    prefetch: B's weights were prefetched right after A's in the weights region during A's turn
+              (Fig. 8(b)); the switch relocates them to the buffer start on the
+              device (Fig. 9 3.b, N1) || A's KV out -> B's KV in; then C's prefetch starts.
+    Latency = switch start -> last (first) layer ready for a per-layer consumer that waits on the
+    weights layer l+1 (and 0) and KV layer l, on the device timeline (CUDA events)."""
+    import aeg_inputs as gi
+    from aeg_inputs import dev as D
+    names = list(descs)
+    shapes = {n: gi.KV_SHAPES[n] for n in names}
+    wsize = {nm: sum(d["rows"] * d["cols"] * 2 + 255 & ~255 for d in descs[nm]) for nm in names}
+    wmax = max(wsize.values())
+    region = wmax + 64 * MIB if mode == "staged" else 2 * wmax + 128 * MIB
+    cfg = aeg.default_config(device_kv_bytes=8 * GIB, host_kv_bytes=8 * GIB, device_weight_bytes=region,
                              kernel=kernel, host_threads=12)
     ctx = aeg.Context(0, cfg)
     kv = {}
     for nm in names:
         sh = shapes[nm]
-        bb = sh[0] * 2 * sh[1] * sh[2] * sh[3] * sh[4]
-        n = GIB // bb
-        hb = ctx.kv_alloc(aeg.POOL_HOST, sh, n)
-        kv[nm] = ("host", hb, n)
+        n = GIB // (sh[0] * 2 * sh[1] * sh[2] * sh[3] * sh[4])
+        kv[nm] = (ctx.kv_alloc(aeg.POOL_HOST, sh, n), n)
     cur = names[0]
-    sh = shapes[cur]
-    db = ctx.kv_alloc(aeg.POOL_DEVICE, sh, kv[cur][2])
-    y = ctx.kv_swap_in(sh, kv[cur][1], db, flags=aeg.FREE_SRC)
+    db = ctx.kv_alloc(aeg.POOL_DEVICE, shapes[cur], kv[cur][1])
+    y = ctx.kv_swap_in(shapes[cur], kv[cur][0], db, flags=aeg.FREE_SRC)
     ctx.layer_ready(y, -1, aeg.READY_BLOCK)
-    kv[cur] = ("dev", db, kv[cur][2])
+    kv[cur] = (db, kv[cur][1])
     offs, x = ctx.weights_stage(descs[cur])
     ctx.layer_ready(x, -1, aeg.READY_BLOCK)
+    pre = None   # (model, xfer, offset of its first tensor)
+    if mode == "prefetch":
+        ctx.weights_reset(-(-wsize[cur] // 256) * 256)
+        o, xp = ctx.weights_stage(descs[names[1]])
+        pre = (names[1], xp, int(o[0]))
     cons = torch.cuda.Stream()
     res = []
-    order = [names[(i + 1) % 3] for i in range(n_switch + 3)]
+    order = [names[(i + 1) % len(names)] for i in range(n_switch + 3)]
     for i, nxt in enumerate(order):
-        prev_sh = shapes[cur]
+        if pre is not None:   # the decode turn of `cur` hides the prefetch (PAPER.md:1365-1368)
+            ctx.layer_ready(pre[1], -1, aeg.READY_BLOCK)
         e0 = torch.cuda.Event(enable_timing=True)
         e0.record(cons)
         ctx.stream_fence(cons.cuda_stream)
-        hb = ctx.kv_alloc(aeg.POOL_HOST, prev_sh, kv[cur][2])
-        xo = ctx.kv_swap_out(prev_sh, kv[cur][1], hb, flags=aeg.FREE_SRC)          # A's KV out (D2H)
-        kv[cur] = ("host", hb, kv[cur][2])
-        ctx.weights_reset(0)
-        _, xw = ctx.weights_stage(descs[nxt])                                       # B's weights in
+        hb = ctx.kv_alloc(aeg.POOL_HOST, shapes[cur], kv[cur][1])
+        xo = ctx.kv_swap_out(shapes[cur], kv[cur][0], hb, flags=aeg.FREE_SRC)        # A's KV out (D2H)
+        kv[cur] = (hb, kv[cur][1])
+        if mode == "staged":
+            ctx.weights_reset(0)
+            _, xw = ctx.weights_stage(descs[nxt])                                      # B's weights in
+            wl = lambda l: min(l, ctx.xfer_layers(xw) - 1)  # noqa: E731
+        else:
+            assert pre[0] == nxt
+            xw = ctx.weights_relocate(pre[2], 0, wsize[nxt])                           # 3.b: on-device copy
+            ctx.xfer_release(pre[1])
+            wl = lambda l: 0  # noqa: E731
         nsh = shapes[nxt]
-        db = ctx.kv_alloc(aeg.POOL_DEVICE, nsh, kv[nxt][2])
-        xi = ctx.kv_swap_in(nsh, kv[nxt][1], db, flags=aeg.FREE_SRC)               # B's KV in
-        kv[nxt] = ("dev", db, kv[nxt][2])
-        L = nsh[0]
+        db = ctx.kv_alloc(aeg.POOL_DEVICE, nsh, kv[nxt][1])
+        xi = ctx.kv_swap_in(nsh, kv[nxt][0], db, flags=aeg.FREE_SRC)                  # B's KV in
+        kv[nxt] = (db, kv[nxt][1])
         ev = []
-        for l in range(L):
-            ctx.layer_ready(xw, min(l + 1, ctx.xfer_layers(xw) - 1), aeg.READY_WAIT_STREAM, cons.cuda_stream)
+        for l in range(nsh[0]):
             if l == 0:
-                ctx.layer_ready(xw, 0, aeg.READY_WAIT_STREAM, cons.cuda_stream)
+                ctx.layer_ready(xw, wl(0), aeg.READY_WAIT_STREAM, cons.cuda_stream)
+            ctx.layer_ready(xw, wl(l + 1), aeg.READY_WAIT_STREAM, cons.cuda_stream)
             ctx.layer_ready(xi, l, aeg.READY_WAIT_STREAM, cons.cuda_stream)
             e = torch.cuda.Event(enable_timing=True)
             e.record(cons)
@@ -483,11 +510,30 @@ def switch_leg(aeg, torch, n_switch, kernel):
         for xx in (xo, xw, xi):
             ctx.layer_ready(xx, -1, aeg.READY_BLOCK)
             ctx.xfer_release(xx)
+        kvb = kv[nxt][1] * nsh[0] * 2 * nsh[1] * nsh[2] * nsh[3] * nsh[4]
         if i >= 3:
-            wbytes = sum(d["rows"] * d["cols"] * 2 for d in descs[nxt])
             res.append(dict(to=nxt, first_ms=e0.elapsed_time(ev[0]), last_ms=e0.elapsed_time(e_end),
-                            bytes_h2d=wbytes + kv[nxt][2] * (nsh[0] * 2 * nsh[1] * nsh[2] * nsh[3] * nsh[4])))
+                            bytes_h2d=(wsize[nxt] if mode == "staged" else 0) + kvb))
+        if i == len(order) - 1:   # bit-exact check of the running model's weights (oracle O8, TP=1)
+            base, _, _ = ctx.weights_region()
+            from oracle import weights as W
+            m = names.index(nxt)
+            bad = 0
+            for k in (0, len(descs[nxt]) // 2, len(descs[nxt]) - 1):
+                d = descs[nxt][k]
+                nb = d["rows"] * d["cols"] * 2
+                o = W.bump_offsets([x["rows"] * x["cols"] * 2 for x in descs[nxt]], 0)[0][k]
+                got = D.read(base + o, min(nb, 1 << 24))
+                exp = gi.region_bytes(gi.w_seed(3), gi.weight_key(m, k), min(nb, 1 << 24))
+                bad += int((got != exp).sum())
         cur = nxt
+        if mode == "prefetch":   # next turn: prefetch the model after `cur` behind it
+            nn = names[(names.index(cur) + 1) % len(names)]
+            ctx.weights_reset(-(-wsize[cur] // 256) * 256)
+            o, xp = ctx.weights_stage(descs[nn])
+            pre = (nn, xp, int(o[0]))
+    if pre is not None:
+        ctx.layer_ready(pre[1], -1, aeg.READY_BLOCK)
     ctx.shutdown()
     per = {}
     for nm in names:
@@ -495,16 +541,16 @@ def switch_leg(aeg, torch, n_switch, kernel):
         if not r:
             continue
         lat = sorted(x["last_ms"] for x in r)
-        wbytes = sum(d["rows"] * d["cols"] * 2 for d in descs[nm])
         per[nm] = {"switches": len(r), "last_layer_ms_p50": round(statistics.median(lat), 2),
                    "last_layer_ms_p90": round(lat[int(0.9 * (len(lat) - 1))], 2),
                    "first_layer_ms_p50": round(statistics.median(x["first_ms"] for x in r), 2),
-                   "h2d_bytes": int(r[0]["bytes_h2d"]), "weights_bytes": int(wbytes),
+                   "h2d_bytes": int(r[0]["bytes_h2d"]), "weights_bytes": int(wsize[nm]),
                    "h2d_GBps": round(r[0]["bytes_h2d"] / (statistics.median(lat) * 1e6), 1),
-                   "eq4_weights_ms_at_64GBps": round(wbytes / (PCIE_NOMINAL * BETA) / 1e6, 1)}
-    return {"workload": "configs[3] 3-model switch (Qwen-1.8B, Llama-7B, Yi-9B shapes), 1 GiB KV each, "
-                        "staged weights through a 2 GiB pinned Stage Buffer", "per_model": per,
-            "model_cache_gen_s": round(gen_s, 1)}
+                   "eq4_weights_ms_at_64GBps": round(wsize[nm] / (PCIE_NOMINAL * BETA) / 1e6, 1)}
+    how = ("weights staged through the 2 GiB pinned Stage Buffer (3.a)" if mode == "staged" else
+           "weights prefetched during the previous turn, relocated on-device at the switch (3.b)")
+    return {"workload": f"configs[3] 3-model switch (Qwen-1.8B, Llama-7B, Yi-9B shapes), 1 GiB KV each; {how}",
+            "per_model": per, "weights_bit_exact_sample": bad == 0}
 
 
 def migrate_leg(aeg, torch, kernel, n_req=4):
@@ -724,7 +770,7 @@ def run_ours(args):
         per_rank = psutil.virtual_memory().available / world
         while n_req > 4 and sum(c2_requests(n_req)[1]) * 8 * MIB * 1.3 > per_rank:
             n_req //= 2
-    sb = SwapBench(aeg, QWEN7B, n_req, kernel).setup()
+    sb = SwapBench(aeg, QWEN7B, n_req, kernel, slot_mib=args.slot_mib, slots=args.slots).setup()
     sb.sink = torch.zeros(1, dtype=torch.int64, device="cuda")
     cons = torch.cuda.Stream()
     bytes_step = 2 * sb.n * sb.sh.block_bytes()
@@ -781,7 +827,15 @@ def run_ours(args):
             mig = migrate_leg_dist(aeg, torch, dist, kernel)
         else:
             mig = migrate_leg(aeg, torch, kernel)
-        sw = None if args.no_switch or world > 1 else switch_leg(aeg, torch, args.switches, kernel)
+        sw = None
+        if not (args.no_switch or world > 1):
+            t0 = time.time()
+            descs, caches = model_caches(["qwen-1.8b", "llama-7b", "yi-9b"])
+            gen_s = time.time() - t0
+            sw = {"staged": switch_leg(aeg, torch, args.switches, kernel, descs, "staged"),
+                  "prefetch": switch_leg(aeg, torch, args.switches, kernel, descs, "prefetch"),
+                  "model_cache_gen_s": round(gen_s, 1)}
+            del caches
         cpu = None if args.no_cpu or rank != 0 else cpu_baseline()
         out.update({"e2e": e2e, "verify": ver, "one_direction": one_dir, "pcie_memcpy_GBps": {k: round(v, 1) for k, v in pc.items()},
                     "switch": sw, "migrate": mig, "cpu_baseline": cpu})
@@ -799,7 +853,8 @@ def run_ours(args):
                        "requests": n_req, "tokens": int(sum(sb.lens)), "blocks": sb.n,
                        "bytes_per_direction": sb.n * sb.sh.block_bytes(), "slab": "1 GiB layer-major",
                        "placement": "device pool aged by seeded churn", "l2": "inputs larger than L2 (32 GiB/step)",
-                       "kernel": args.kernel, "parallelism": f"replicas x{world}"},
+                       "kernel": args.kernel, "staging_slot_mib": sb.cfg.staging_slot_bytes >> 20,
+                       "staging_slots": sb.cfg.staging_slots, "parallelism": f"replicas x{world}"},
             "roofline": {"bound": "hbm", "kernel": "gather (swap-out, H2)", "achieved": round(g_ach, 1),
                          "peak": hbm, "peak_source": hbm_src, "unit": "GB/s",
                          "frac": round(g_ach / hbm, 3), "traffic": ncu_traffic("gather"),
