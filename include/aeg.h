@@ -138,7 +138,7 @@ typedef struct {
 /* ---- lifecycle -------------------------------------------------------------------------- */
 
 /* Fill *cfg with defaults: 1 GiB slabs (layer-major), 2 GiB stage ring of 64 MiB chunks,
- * 4 x 128 MiB staging slots per direction, 8 host threads, AUTO kernels; region sizes 0.
+ * 3 x 1 GiB staging slots per direction, 8 host threads, AUTO kernels (BULK); region sizes 0.
  * Returns AEG_OK. */
 int aeg_config_default(aeg_config* cfg);
 
@@ -249,8 +249,9 @@ int aeg_weights_stage(aeg_ctx ctx, const aeg_weight_desc* descs, int32_t n, int3
                       int32_t tp_size, uint64_t* dev_offsets_out, aeg_xfer* out);
 
 /* Reset the bump pointer to `offset` (0 = region base): "deallocations can be done instantly by
- * simply resetting that pointer".  STATE while a weight transfer is in
- * flight. */
+ * simply resetting that pointer".  Does not wait: later staging and
+ * relocation run on the same weights stream, so they are ordered after earlier ones.  INVALID for
+ * an offset beyond the region or not 256-byte aligned. */
 int aeg_weights_reset(aeg_ctx ctx, uint64_t offset);
 
 /* Current bump pointer, base pointer and size of the weights region. */

@@ -78,8 +78,8 @@ int aeg_config_default(aeg_config* cfg) {
     cfg->host_slab_bytes = 1ull << 30;
     cfg->stage_ring_bytes = 2ull << 30;  // "Stage Buffer (2 GB)"
     cfg->stage_chunk_bytes = 64ull << 20;
-    cfg->staging_slot_bytes = 128ull << 20;
-    cfg->staging_slots = 4;
+    cfg->staging_slot_bytes = 1ull << 30;  // one launch per layer for 7B-class batches (profiles/r01)
+    cfg->staging_slots = 3;
     cfg->table_arena_bytes = 64ull << 20;
     cfg->host_threads = 8;
     cfg->dev_slab_layout = AEG_LAYER_MAJOR;

@@ -2,6 +2,8 @@
 // table arena, kernel timing and the primitive trace.
 #include "engine.h"
 
+#include <sys/mman.h>
+
 #include <algorithm>
 #include <chrono>
 #include <cinttypes>
@@ -10,8 +12,40 @@
 namespace aeg {
 
 namespace {
-constexpr uint64_t kMiB = 1ull << 20, kGiB = 1ull << 30;
+constexpr uint64_t kMiB = 1ull << 20;
 constexpr uint64_t kAlign = 2 * kMiB;
+
+// Page-lock `bytes` of host memory once at init.  cudaHostAlloc faults and
+// pins pages on one thread (~2.5 GB/s measured on the B200 box); instead: anonymous mmap with
+// transparent huge pages, first touch from several threads, then cudaHostRegister of the populated
+// range (~19 GB/s measured, same DMA bandwidth) — 41 GiB pin in ~2 s instead of ~17 s.
+char* pin_host(uint64_t bytes) {
+  void* p = mmap(nullptr, bytes, PROT_READ | PROT_WRITE, MAP_PRIVATE | MAP_ANONYMOUS, -1, 0);
+  AEG_REQUIRE(p != MAP_FAILED, AEG_ERR_OOM, "mmap of %llu host bytes failed", (unsigned long long)bytes);
+  madvise(p, bytes, MADV_HUGEPAGE);
+  char* b = static_cast<char*>(p);
+  const unsigned T = std::max(1u, std::min(16u, std::thread::hardware_concurrency()));
+  std::vector<std::thread> th;
+  for (unsigned i = 0; i < T; ++i)
+    th.emplace_back([=] {
+      for (uint64_t o = bytes * i / T / 4096 * 4096; o < bytes * (i + 1) / T; o += 4096) b[o] = 0;
+    });
+  for (auto& t : th) t.join();
+  cudaError_t e = cudaHostRegister(b, bytes, cudaHostRegisterPortable | cudaHostRegisterMapped);
+  if (e != cudaSuccess) {
+    munmap(b, bytes);
+    fail(AEG_ERR_CUDA, "cudaHostRegister of %llu bytes failed: %s", (unsigned long long)bytes, cudaGetErrorString(e));
+  }
+  void* dp = nullptr;
+  CUDA_TRY(cudaHostGetDevicePointer(&dp, b, 0));
+  AEG_REQUIRE(dp == b, AEG_ERR_CUDA, "registered host memory is not addressable at the same pointer on the device");
+  return b;
+}
+
+void unpin_host(char* b, uint64_t bytes) {
+  cudaHostUnregister(b);
+  munmap(b, bytes);
+}
 }  // namespace
 
 // ------------------------------------------------------------------------------------ init
@@ -54,8 +88,7 @@ void Ctx::init(int dev, const aeg_config& c) {
   const uint64_t hkv = align_up(cfg.host_kv_bytes, kAlign);
   const uint64_t hst = align_up(cfg.stage_ring_bytes, kAlign);
   host_mem_bytes = hkv + hst + tab;
-  CUDA_TRY(cudaHostAlloc(reinterpret_cast<void**>(&host_mem), host_mem_bytes,
-                         cudaHostAllocPortable | cudaHostAllocMapped));
+  host_mem = pin_host(host_mem_bytes);
   host_kv = host_mem;
   host_stage = host_mem + hkv;
   tables.host = host_stage + hst;
@@ -127,7 +160,7 @@ void Ctx::shutdown() {
   for (cudaStream_t s : {s_gather, s_d2h, s_h2d, s_scatter, s_weights, s_migrate})
     if (s) cudaStreamDestroy(s);
   if (dev_mem) cudaFree(dev_mem);
-  if (host_mem) cudaFreeHost(host_mem);
+  if (host_mem) unpin_host(host_mem, host_mem_bytes);
 }
 
 // ------------------------------------------------------------------------------- daemon ⑧

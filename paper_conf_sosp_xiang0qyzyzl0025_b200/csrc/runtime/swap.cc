@@ -112,7 +112,10 @@ static void host_dmas(Ctx& c, const Shape& sh, const std::vector<Run>& runs, con
   }
 }
 
-static int impl_of(const aeg_config& cfg) { return cfg.kernel == AEG_KERNEL_BULK ? IMPL_BULK : IMPL_LSU; }
+// AUTO = BULK (cp.async.bulk through shared memory): measured 5.93 TB/s in-step for the C2 gather vs
+// 5.56 TB/s for LSU with 1 GiB slots (profiles/r01).  Stores into another GPU's pool use LSU under AUTO
+// (plain st.global to peer addresses) unless BULK is requested explicitly.
+static int impl_of(const aeg_config& cfg) { return cfg.kernel == AEG_KERNEL_LSU ? IMPL_LSU : IMPL_BULK; }
 
 // ----------------------------------------------------------------------------- swap-out H3
 uint64_t Ctx::swap_out(const Shape& sh, const aeg_block* dev, const aeg_block* host, int32_t n, uint32_t flags) {
@@ -288,7 +291,8 @@ uint64_t Ctx::migrate(const Shape& sh, const aeg_block* src, int32_t peer, const
   const uint64_t layer = uint64_t(n) * sh.chunk();
   int32_t lps = 1;
   if (n > 0 && layer < kPackLayerBytes) lps = int32_t(std::min<uint64_t>(sh.L, std::max<uint64_t>(1, kPackLayerBytes / layer)));
-  const int impl = impl_of(cfg);
+  const int impl = (P && !P->same_process && cfg.kernel == AEG_KERNEL_AUTO) || (P && P->device != device && cfg.kernel == AEG_KERNEL_AUTO)
+                       ? IMPL_LSU : impl_of(cfg);
   for (int32_t la = 0; la < sh.L; la += lps) {
     const int32_t lb = std::min(sh.L, la + lps);
     if (n > 0) {

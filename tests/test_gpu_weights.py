@@ -120,11 +120,16 @@ def test_relocate_is_memmove():
         ctx.layer_ready(x, -1, aeg.READY_BLOCK)            # the prefetch has landed
         _, _, end = ctx.weights_region()
         size = end - running
-        before = D.read(base, end)
-        y = ctx.weights_relocate(running, 0, size)           # overlapping move (size > gap)
+        assert size > running                                 # overlapping move (size > gap)
+        y = ctx.weights_relocate(running, 0, size)
         ctx.layer_ready(y, -1, aeg.READY_BLOCK)
+        # expected: oracle O8 staging at base `running`, then oracle N1 memmove to 0
+        img, offs_o, end_o = W.stage(tens, descs, 0, 1, region_bytes=wbytes, base=running)
+        assert end_o == end and [int(o) for o in offs] == offs_o
+        from oracle.memmove import memmove
+        exp = memmove(img, running, 0, size)
         got = D.read(base, size)
-        assert first_diff(got, before[running:end]) is None
+        assert first_diff(got, exp[:size]) is None
         ctx.xfer_release(x)
         ctx.xfer_release(y)
     finally:

@@ -23,6 +23,8 @@ MUTANTS = [
     ("oracle/weights.py", "return w[:, r * part:(r + 1) * part]", "return w[:, r:(r + 1) * part]"),
     ("oracle/weights.py", "for gi in range(groups)], axis=0)", "for gi in range(groups)][::-1], axis=0)"),
     ("oracle/weights.py", "p = align_up(p + n)", "p = p + n"),
+    ("oracle/memmove.py", "out[dst:dst + n] = tmp", "out[dst:dst + n] = tmp[::-1]"),
+    ("oracle/memmove.py", "tmp = buf[src:src + n].copy()", "tmp = buf[dst:dst + n].copy()"),
     ("oracle/rules.py", "pending.setdefault(e[1], set()).add(c)", "pass"),
     ("oracle/rules.py", "captured[e[2]] = tail.get(e[1])", "captured[e[2]] = len(ops) - 1 if ops else None"),
 ]
@@ -41,7 +43,7 @@ def main():
             open(f, "w").write(src.replace(old, new, 1))
             r = subprocess.run([sys.executable, "-m", "pytest", "-x", "-q", "-p", "no:cacheprovider",
                                 "tests/test_oracle_shape.py", "tests/test_oracle_slab.py", "tests/test_oracle_kv.py",
-                                "tests/test_oracle_weights.py", "tests/test_oracle_rules.py"],
+                                "tests/test_oracle_weights.py", "tests/test_oracle_rules.py", "tests/test_oracle_memmove.py"],
                                cwd=d, capture_output=True, text=True)
             status = "killed" if r.returncode != 0 else "SURVIVED"
             print(f"{status:9s} {path}: {new[:70]!r}")
