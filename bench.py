@@ -81,13 +81,24 @@ class Dist:
         import torch
         self.world, self.rank, self.local = world, rank, local
         self.torch = torch
-        torch.cuda.set_device(local)
+        # one process per GPU; AEG_DIST_BACKEND=gloo lets several ranks share one GPU to exercise the
+        # multi-rank path on a 1-GPU box (control data only travels through torch.distributed)
+        self.backend = os.environ.get("AEG_DIST_BACKEND", "nccl")
+        self.device = local % max(1, torch.cuda.device_count())
+        torch.cuda.set_device(self.device)
         self.pg = None
         if world > 1:
             import torch.distributed as td
             os.environ.setdefault("MASTER_ADDR", "127.0.0.1")
-            td.init_process_group("nccl", device_id=torch.device("cuda", local))
+            if self.backend == "nccl":
+                td.init_process_group("nccl", device_id=torch.device("cuda", self.device))
+            else:
+                td.init_process_group(self.backend)
             self.td = td
+
+    def _t(self, v):
+        dev = "cuda" if self.backend == "nccl" else "cpu"
+        return self.torch.tensor([v], dtype=self.torch.float64, device=dev)
 
     def barrier(self):
         self.torch.cuda.synchronize()
@@ -97,14 +108,14 @@ class Dist:
     def max(self, v: float) -> float:
         if self.world == 1:
             return v
-        t = self.torch.tensor([v], dtype=self.torch.float64, device="cuda")
+        t = self._t(v)
         self.td.all_reduce(t, op=self.td.ReduceOp.MAX)
         return float(t.item())
 
     def sum(self, v: float) -> float:
         if self.world == 1:
             return v
-        t = self.torch.tensor([v], dtype=self.torch.float64, device="cuda")
+        t = self._t(v)
         self.td.all_reduce(t, op=self.td.ReduceOp.SUM)
         return float(t.item())
 
@@ -219,7 +230,8 @@ class SwapBench:
             cfg.staging_slots = slots
         self.cfg = cfg
         t0 = time.time()
-        self.ctx = aeg.Context(0, cfg)
+        import torch
+        self.ctx = aeg.Context(torch.cuda.current_device(), cfg)
         self.init_s = time.time() - t0
         self.dg = OK.PoolGeom(cfg.device_kv_bytes, GIB, aeg.LAYER_MAJOR)
         self.hg = OK.PoolGeom(cfg.host_kv_bytes, GIB, aeg.LAYER_MAJOR)
@@ -433,7 +445,7 @@ def model_caches(names):
     return descs, caches
 
 
-def switch_leg(aeg, torch, n_switch, kernel, descs, mode="staged"):
+def switch_leg(aeg, torch, n_switch, kernel, descs, mode="staged", caches=None):
     """configs[3]: token-level switch among Qwen-1.8B / Llama-7B / Yi-9B shapes on one GPU.
     staged  : switch(A->B) = swap-out of A's 1 GiB decode KV (D2H) || staging of B's weights through
               the pinned Stage Buffer (H2D, Fig. 9 3.a) -> swap-in of B's KV.
@@ -452,6 +464,12 @@ def switch_leg(aeg, torch, n_switch, kernel, descs, mode="staged"):
     cfg = aeg.default_config(device_kv_bytes=8 * GIB, host_kv_bytes=8 * GIB, device_weight_bytes=region,
                              kernel=kernel, host_threads=12)
     ctx = aeg.Context(0, cfg)
+    reg_s = None
+    if mode == "direct":   # page-lock the Model Caches once ("no pinning during scaling")
+        t0 = time.time()
+        for nm in names:
+            ctx.host_register(caches[nm].ctypes.data, caches[nm].nbytes)
+        reg_s = time.time() - t0
     kv = {}
     for nm in names:
         sh = shapes[nm]
@@ -481,7 +499,7 @@ def switch_leg(aeg, torch, n_switch, kernel, descs, mode="staged"):
         hb = ctx.kv_alloc(aeg.POOL_HOST, shapes[cur], kv[cur][1])
         xo = ctx.kv_swap_out(shapes[cur], kv[cur][0], hb, flags=aeg.FREE_SRC)        # A's KV out (D2H)
         kv[cur] = (hb, kv[cur][1])
-        if mode == "staged":
+        if mode in ("staged", "direct"):
             ctx.weights_reset(0)
             _, xw = ctx.weights_stage(descs[nxt])                                      # B's weights in
             wl = lambda l: min(l, ctx.xfer_layers(xw) - 1)  # noqa: E731
@@ -513,7 +531,7 @@ def switch_leg(aeg, torch, n_switch, kernel, descs, mode="staged"):
         kvb = kv[nxt][1] * nsh[0] * 2 * nsh[1] * nsh[2] * nsh[3] * nsh[4]
         if i >= 3:
             res.append(dict(to=nxt, first_ms=e0.elapsed_time(ev[0]), last_ms=e0.elapsed_time(e_end),
-                            bytes_h2d=(wsize[nxt] if mode == "staged" else 0) + kvb))
+                            bytes_h2d=(0 if mode == "prefetch" else wsize[nxt]) + kvb))
         if i == len(order) - 1:   # bit-exact check of the running model's weights (oracle O8, TP=1)
             base, _, _ = ctx.weights_region()
             from oracle import weights as W
@@ -546,11 +564,14 @@ def switch_leg(aeg, torch, n_switch, kernel, descs, mode="staged"):
                    "first_layer_ms_p50": round(statistics.median(x["first_ms"] for x in r), 2),
                    "h2d_bytes": int(r[0]["bytes_h2d"]), "weights_bytes": int(wsize[nm]),
                    "h2d_GBps": round(r[0]["bytes_h2d"] / (statistics.median(lat) * 1e6), 1),
-                   "eq4_weights_ms_at_64GBps": round(wsize[nm] / (PCIE_NOMINAL * BETA) / 1e6, 1)}
-    how = ("weights staged through the 2 GiB pinned Stage Buffer (3.a)" if mode == "staged" else
-           "weights prefetched during the previous turn, relocated on-device at the switch (3.b)")
+                   "eq4_weights_ms_at_64GBps": round(wsize[nm] / (PCIE_NOMINAL * BETA) / 1e6, 1),
+                   # N4: Eq. 4 solved for beta on this B200: T = size / (BW * beta)
+                   "eq4_beta_fit": round(wsize[nm] / (PCIE_NOMINAL * 1e9 * statistics.median(lat) / 1e3), 3)}
+    how = {"staged": "weights staged through the 2 GiB pinned Stage Buffer by host threads (3.a)",
+           "direct": "weights DMA'd straight from the page-locked Model Cache (registered once)",
+           "prefetch": "weights prefetched during the previous turn, relocated on-device at the switch (3.b)"}[mode]
     return {"workload": f"configs[3] 3-model switch (Qwen-1.8B, Llama-7B, Yi-9B shapes), 1 GiB KV each; {how}",
-            "per_model": per, "weights_bit_exact_sample": bad == 0}
+            "per_model": per, "weights_bit_exact_sample": bad == 0, "register_s": reg_s}
 
 
 def migrate_leg(aeg, torch, kernel, n_req=4):
@@ -631,7 +652,7 @@ def migrate_leg_dist(aeg, torch, dist, kernel, n_req=4):
     cfg = aeg.default_config(device_kv_bytes=nslab * slab, host_kv_bytes=GIB, dev_slab_bytes=slab,
                              dev_slab_layout=aeg.LAYER_MAJOR if PD.role(rank, world) == "prefill" else aeg.BLOCK_MAJOR,
                              kernel=kernel, flags=aeg.CFG_TIMING)
-    ctx = aeg.Context(dist.local, cfg)
+    ctx = aeg.Context(dist.device, cfg)
     geom = OK.PoolGeom(nslab * slab, slab, cfg.dev_slab_layout)
     base, _ = ctx.pool_region(0)
     seed = gi.kv_seed(3)
@@ -779,7 +800,7 @@ def run_ours(args):
         sb.step(torch, cons)
     sb.ctx.kernel_stats_reset()
     dist.barrier()
-    with Clocks(local) as clk:
+    with Clocks(dist.device) as clk:
         e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         e0.record(cons)
         for _ in range(args.steps):
@@ -834,6 +855,7 @@ def run_ours(args):
             gen_s = time.time() - t0
             sw = {"staged": switch_leg(aeg, torch, args.switches, kernel, descs, "staged"),
                   "prefetch": switch_leg(aeg, torch, args.switches, kernel, descs, "prefetch"),
+                  "direct": switch_leg(aeg, torch, args.switches, kernel, descs, "direct", caches),
                   "model_cache_gen_s": round(gen_s, 1)}
             del caches
         cpu = None if args.no_cpu or rank != 0 else cpu_baseline()
