@@ -74,7 +74,9 @@ enum { AEG_SPLIT_REPLICATED = 0, AEG_SPLIT_COL = 1, AEG_SPLIT_ROW = 2, AEG_SPLIT
 enum {
   AEG_CFG_HOST_ONLY = 1u << 0, /* no CUDA at all: allocator / bookkeeping only (CPU tests)   */
   AEG_CFG_NO_DAEMON = 1u << 1, /* no reclaim thread: reclaim only via aeg_reclaim            */
-  AEG_CFG_TIMING = 1u << 2     /* time every gather/scatter/migrate launch with CUDA events  */
+  AEG_CFG_TIMING = 1u << 2,    /* time every gather/scatter/migrate launch with CUDA events  */
+  AEG_CFG_SHARED_HOST = 1u << 3 /* CPU KV region in POSIX shared memory, mappable by peers:
+                                   the node-shared "Unified CPU KV Cache" (Fig. 5) */
 };
 /* kernel selection for gather/scatter/migrate (AEG_KERNEL_AUTO picks the measured best) */
 enum { AEG_KERNEL_AUTO = 0, AEG_KERNEL_LSU = 1, AEG_KERNEL_BULK = 2 };
@@ -215,6 +217,21 @@ int aeg_kv_swap_in(aeg_ctx ctx, const aeg_kv_shape* shape, const aeg_block* host
  * AEG_FREE_SRC frees the source blocks. */
 int aeg_kv_migrate(aeg_ctx ctx, const aeg_kv_shape* shape, const aeg_block* src, int32_t peer,
                    const aeg_block* dst, int32_t n, uint32_t flags, aeg_xfer* out);
+
+/* Paper route P->C->D (Fig. 10 ③④⑤; NEXT-2): swap-in from ANOTHER process's
+ * shared CPU KV region (the peer exported with AEG_CFG_SHARED_HOST; `peer` as given to
+ * aeg_import_peer, or -1 for this context's own host pool).  Layer l's H2D waits on layer l of
+ * transfer `after` (0 = none) — typically the peer's swap-out imported with aeg_xfer_import (rule ❷
+ * across instances via IPC events).  peer_host handles are validated against
+ * the peer's geometry only; ownership stays with the peer, which frees them with aeg_kv_free_after
+ * on this transfer (rule ❸).  Otherwise as aeg_kv_swap_in (AEG_FREE_SRC is INVALID for a peer). */
+int aeg_kv_swap_in_from(aeg_ctx ctx, const aeg_kv_shape* shape, int32_t peer, const aeg_block* peer_host,
+                        const aeg_block* dev, int32_t n, aeg_xfer after, uint32_t flags, aeg_xfer* out);
+
+/* Free owned blocks that a transfer `after` (local or imported) still reads or writes: they go to
+ * the move list until `after` completes (step ⑧), e.g. the prefill instance's
+ * CPU blocks after the decode instance's swap-in of them was imported. */
+int aeg_kv_free_after(aeg_ctx ctx, int32_t pool, const aeg_block* blocks, int32_t n, aeg_xfer after);
 
 /* Order every later transfer of this context after the work currently enqueued on `cuda_stream`
  * (a cudaStream_t; NULL = legacy default stream), e.g. the prefill kernels that wrote the blocks. */

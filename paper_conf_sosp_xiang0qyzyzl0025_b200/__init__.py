@@ -25,7 +25,7 @@ OK, NOT_READY, ERR_INVALID, ERR_OOM, ERR_CUDA, ERR_STATE = 0, 1, -1, -2, -3, -4
 READY_QUERY, READY_WAIT_STREAM, READY_BLOCK = 0, 1, 2
 FREE_SRC, NO_DEPS = 1, 2
 SPLIT_REPLICATED, SPLIT_COL, SPLIT_ROW, SPLIT_VOCAB = 0, 1, 2, 3
-CFG_HOST_ONLY, CFG_NO_DAEMON, CFG_TIMING = 1, 2, 4
+CFG_HOST_ONLY, CFG_NO_DAEMON, CFG_TIMING, CFG_SHARED_HOST = 1, 2, 4, 8
 KERNEL_AUTO, KERNEL_LSU, KERNEL_BULK = 0, 1, 2
 K_GATHER, K_SCATTER, K_MIGRATE, K_RELOCATE = 0, 1, 2, 3
 
@@ -100,6 +100,8 @@ _SIGS = {
     "aeg_kv_swap_out": [P, C.POINTER(KVShape), PU64, PU64, I32, U32, PU64],
     "aeg_kv_swap_in": [P, C.POINTER(KVShape), PU64, PU64, I32, U32, PU64],
     "aeg_kv_migrate": [P, C.POINTER(KVShape), PU64, I32, PU64, I32, U32, PU64],
+    "aeg_kv_swap_in_from": [P, C.POINTER(KVShape), I32, PU64, PU64, I32, U64, U32, PU64],
+    "aeg_kv_free_after": [P, I32, PU64, I32, U64],
     "aeg_stream_fence": [P, P],
     "aeg_layer_ready": [P, U64, I32, I32, P],
     "aeg_xfer_layers": [P, U64, PI32],
@@ -250,6 +252,19 @@ class Context:
         sh = KVShape.of(shape)
         _chk(lib().aeg_kv_migrate(self.h, C.byref(sh), _p64(s), int(peer), _p64(d), int(s.size), flags, C.byref(x)))
         return x.value
+
+    def kv_swap_in_from(self, shape, peer: int, peer_host, dev, after: int = 0, flags: int = 0) -> int:
+        h, d = _blocks(peer_host), _blocks(dev)
+        assert d.size == h.size
+        x = C.c_uint64()
+        sh = KVShape.of(shape)
+        _chk(lib().aeg_kv_swap_in_from(self.h, C.byref(sh), int(peer), _p64(h), _p64(d), int(d.size), int(after),
+                                       flags, C.byref(x)))
+        return x.value
+
+    def kv_free_after(self, pool: int, blocks, after: int):
+        b = _blocks(blocks)
+        _chk(lib().aeg_kv_free_after(self.h, pool, _p64(b), int(b.size), int(after)))
 
     def stream_fence(self, stream: int = 0):
         _chk(lib().aeg_stream_fence(self.h, P(stream)))

@@ -54,6 +54,10 @@ struct IpcBlob {
   uint64_t pool_bytes, slab_bytes;
   int32_t layout, pad;
   cudaIpcMemHandle_t mem;
+  // shared CPU KV region (AEG_CFG_SHARED_HOST), empty name if none
+  char shm[64];
+  uint64_t host_bytes, host_slab_bytes, host_kv_bytes;
+  int32_t host_layout, pad2;
 };
 
 struct XferBlobHead {
@@ -255,6 +259,31 @@ int aeg_kv_migrate(aeg_ctx ctx, const aeg_kv_shape* shape, const aeg_block* src,
   });
 }
 
+int aeg_kv_swap_in_from(aeg_ctx ctx, const aeg_kv_shape* shape, int32_t peer, const aeg_block* peer_host,
+                        const aeg_block* dev, int32_t n, aeg_xfer after, uint32_t flags, aeg_xfer* out) {
+  return guarded([&] {
+    Ctx& c = C(ctx);
+    AEG_REQUIRE(out, AEG_ERR_INVALID, "out is NULL");
+    const aeg::Shape sh = aeg::Shape::from(shape);
+    std::lock_guard<std::mutex> g(c.mu);
+    set_device(c);
+    *out = c.swap_in_from(sh, peer, peer_host, dev, n, after, flags);
+    return AEG_OK;
+  });
+}
+
+int aeg_kv_free_after(aeg_ctx ctx, int32_t pool, const aeg_block* blocks, int32_t n, aeg_xfer after) {
+  return guarded([&] {
+    Ctx& c = C(ctx);
+    AEG_REQUIRE(pool == AEG_POOL_DEVICE || pool == AEG_POOL_HOST, AEG_ERR_INVALID, "bad pool %d", pool);
+    std::lock_guard<std::mutex> g(c.mu);
+    set_device(c);
+    c.poll();
+    c.pool[pool].free_after(blocks, n, after);
+    return AEG_OK;
+  });
+}
+
 int aeg_stream_fence(aeg_ctx ctx, void* stream) {
   return guarded([&] {
     Ctx& c = C(ctx);
@@ -398,6 +427,13 @@ int aeg_export_ipc(aeg_ctx ctx, void* buf, uint64_t* len) {
     b.slab_bytes = c.pool[AEG_POOL_DEVICE].slab_bytes;
     b.layout = c.pool[AEG_POOL_DEVICE].layout;
     CUDA_TRY(cudaIpcGetMemHandle(&b.mem, c.dev_mem));
+    if (!c.shm_name.empty()) {
+      std::snprintf(b.shm, sizeof b.shm, "%s", c.shm_name.c_str());
+      b.host_bytes = c.host_kv_mapped;
+      b.host_kv_bytes = c.pool[AEG_POOL_HOST].pool_bytes;
+      b.host_slab_bytes = c.pool[AEG_POOL_HOST].slab_bytes;
+      b.host_layout = c.pool[AEG_POOL_HOST].layout;
+    }
     std::memcpy(buf, &b, sizeof b);
     *len = sizeof b;
     return AEG_OK;
@@ -437,10 +473,18 @@ int aeg_import_peer(aeg_ctx ctx, int32_t peer, const void* buf, uint64_t len) {
       p->ipc_base = static_cast<char*>(ptr);
       p->dev_kv = p->ipc_base;  // dev_kv is the start of the exporter's allocation
     }
+    if (b.shm[0] && !p->same_process) {  // the peer's part of the node-shared CPU KV cache
+      b.shm[sizeof b.shm - 1] = 0;
+      p->host_kv = aeg::map_shared_host(b.shm, b.host_bytes, false);
+      p->host_bytes = b.host_bytes;
+      p->host_geom.init(AEG_POOL_HOST, b.host_kv_bytes, b.host_slab_bytes, b.host_layout);
+      p->has_host = true;
+    }
     p->valid = true;
     auto it = c.peers.find(peer);
     if (it != c.peers.end()) {
       if (it->second->ipc_base) cudaIpcCloseMemHandle(it->second->ipc_base);
+      if (it->second->has_host) aeg::unmap_shared_host(it->second->host_kv, it->second->host_bytes);
       p->events = std::move(it->second->events);
     }
     c.peers[peer] = std::move(p);

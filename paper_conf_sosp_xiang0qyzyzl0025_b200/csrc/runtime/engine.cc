@@ -2,7 +2,9 @@
 // table arena, kernel timing and the primitive trace.
 #include "engine.h"
 
+#include <fcntl.h>
 #include <sys/mman.h>
+#include <unistd.h>
 
 #include <algorithm>
 #include <chrono>
@@ -46,7 +48,54 @@ void unpin_host(char* b, uint64_t bytes) {
   cudaHostUnregister(b);
   munmap(b, bytes);
 }
+
+void touch(char* b, uint64_t bytes) {
+  const unsigned T = std::max(1u, std::min(16u, std::thread::hardware_concurrency()));
+  std::vector<std::thread> th;
+  for (unsigned i = 0; i < T; ++i)
+    th.emplace_back([=] {
+      for (uint64_t o = bytes * i / T / 4096 * 4096; o < bytes * (i + 1) / T; o += 4096) b[o] = 0;
+    });
+  for (auto& t : th) t.join();
+}
+
+void register_same_ptr(char* b, uint64_t bytes) {
+  CUDA_TRY(cudaHostRegister(b, bytes, cudaHostRegisterPortable | cudaHostRegisterMapped));
+  void* dp = nullptr;
+  CUDA_TRY(cudaHostGetDevicePointer(&dp, b, 0));
+  AEG_REQUIRE(dp == b, AEG_ERR_CUDA, "registered host memory is not addressable at the same pointer on the device");
+}
 }  // namespace
+
+// The node-shared Unified CPU KV Cache (Fig. 5; NEXT-2): a POSIX shared-memory object
+// mapped by every instance of the node, page-locked once per process.
+char* map_shared_host(const std::string& name, uint64_t bytes, bool create) {
+  int fd = shm_open(name.c_str(), create ? (O_CREAT | O_EXCL | O_RDWR) : O_RDWR, 0600);
+  AEG_REQUIRE(fd >= 0, AEG_ERR_INVALID, "shm_open(%s) failed", name.c_str());
+  if (create && ftruncate(fd, off_t(bytes)) != 0) {
+    close(fd);
+    shm_unlink(name.c_str());
+    fail(AEG_ERR_OOM, "ftruncate of shared host region %s failed", name.c_str());
+  }
+  void* p = mmap(nullptr, bytes, PROT_READ | PROT_WRITE, MAP_SHARED, fd, 0);
+  close(fd);
+  AEG_REQUIRE(p != MAP_FAILED, AEG_ERR_OOM, "mmap of shared host region %s failed", name.c_str());
+  char* b = static_cast<char*>(p);
+  if (create) touch(b, bytes);
+  try {
+    register_same_ptr(b, bytes);
+  } catch (...) {
+    munmap(b, bytes);
+    if (create) shm_unlink(name.c_str());
+    throw;
+  }
+  return b;
+}
+
+void unmap_shared_host(char* b, uint64_t bytes) {
+  cudaHostUnregister(b);
+  munmap(b, bytes);
+}
 
 // ------------------------------------------------------------------------------------ init
 void Ctx::init(int dev, const aeg_config& c) {
@@ -87,10 +136,20 @@ void Ctx::init(int dev, const aeg_config& c) {
   // One pinned host allocation, pinned once: [CPU KV | Stage Buffer | tables]
   const uint64_t hkv = align_up(cfg.host_kv_bytes, kAlign);
   const uint64_t hst = align_up(cfg.stage_ring_bytes, kAlign);
-  host_mem_bytes = hkv + hst + tab;
-  host_mem = pin_host(host_mem_bytes);
-  host_kv = host_mem;
-  host_stage = host_mem + hkv;
+  if (cfg.flags & AEG_CFG_SHARED_HOST) {
+    static std::atomic<int> seq{0};
+    shm_name = "/aegkv." + std::to_string(getpid()) + "." + std::to_string(seq++);
+    host_kv = map_shared_host(shm_name, hkv, true);
+    host_kv_mapped = hkv;
+    host_mem_bytes = hst + tab;
+    host_mem = pin_host(host_mem_bytes);
+    host_stage = host_mem;
+  } else {
+    host_mem_bytes = hkv + hst + tab;
+    host_mem = pin_host(host_mem_bytes);
+    host_kv = host_mem;
+    host_stage = host_mem + hkv;
+  }
   tables.host = host_stage + hst;
 
   int lo = 0, hi = 0;
@@ -154,6 +213,11 @@ void Ctx::shutdown() {
     Peer* p = kv.second.get();
     for (auto& e : p->events) cudaEventDestroy(e.second);
     if (p->ipc_base) cudaIpcCloseMemHandle(p->ipc_base);
+    if (p->has_host) unmap_shared_host(p->host_kv, p->host_bytes);
+  }
+  if (!shm_name.empty()) {
+    unmap_shared_host(host_kv, host_kv_mapped);
+    shm_unlink(shm_name.c_str());
   }
   for (auto& r : registered) cudaHostUnregister(r.first);
   cudaEventDestroy(fence_ev);

@@ -28,6 +28,10 @@ namespace aeg {
 
 enum XferKind { X_SWAP_OUT = 0, X_SWAP_IN, X_MIGRATE, X_WEIGHTS, X_RELOCATE, X_DEBUG, X_IMPORTED };
 
+// Shared (node-wide) CPU KV region: create (exporter) or map (importer), page-locked (engine.cc).
+char* map_shared_host(const std::string& name, uint64_t bytes, bool create);
+void unmap_shared_host(char* b, uint64_t bytes);
+
 // One transfer: one CUDA event per readiness layer (reading 11) + one completion event.
 struct Xfer {
   uint64_t id = 0;
@@ -77,6 +81,11 @@ struct Peer {
   char* ipc_base = nullptr;        // what cudaIpcOpenMemHandle returned (to close)
   SlabPool geom;                   // geometry only (no ownership state)
   std::unordered_map<std::string, cudaEvent_t> events;  // opened IPC events, by handle bytes
+  // the peer's shared CPU KV region (AEG_CFG_SHARED_HOST), mapped + page-locked here
+  char* host_kv = nullptr;
+  uint64_t host_bytes = 0;
+  SlabPool host_geom;
+  bool has_host = false;
 };
 
 struct KStat {
@@ -108,6 +117,8 @@ struct Ctx {
   uint64_t host_mem_bytes = 0;
   char* host_kv = nullptr;
   char* host_stage = nullptr;
+  std::string shm_name;   // AEG_CFG_SHARED_HOST: POSIX shm object holding the CPU KV region
+  uint64_t host_kv_mapped = 0;
   uint64_t w_bump = 0;
   int w_inflight = 0;
 
@@ -175,6 +186,9 @@ struct Ctx {
   // ---- data paths (swap.cc, weights.cc)
   uint64_t swap_out(const Shape& sh, const aeg_block* dev, const aeg_block* host, int32_t n, uint32_t flags);
   uint64_t swap_in(const Shape& sh, const aeg_block* host, const aeg_block* dev, int32_t n, uint32_t flags);
+  // swap-in from a (possibly peer) host region with an extra per-layer dependency `after` (NEXT-2)
+  uint64_t swap_in_from(const Shape& sh, int32_t peer, const aeg_block* host, const aeg_block* dev, int32_t n,
+                        uint64_t after, uint32_t flags);
   uint64_t migrate(const Shape& sh, const aeg_block* src, int32_t peer, const aeg_block* dst, int32_t n,
                    uint32_t flags);
   uint64_t relocate(uint64_t src_off, uint64_t dst_off, uint64_t bytes);

@@ -152,6 +152,26 @@ void SlabPool::free(const aeg_block* b, int32_t n) {
   for (uint32_t s : touched) maybe_unassign(s);
 }
 
+void SlabPool::free_after(const aeg_block* b, int32_t n, uint64_t x) {
+  check_owned(b, n, nullptr);
+  if (!x || is_done(x)) {
+    free(b, n);
+    return;
+  }
+  for (int32_t i = 0; i < n; ++i) {
+    const uint32_t s = block_slab(b[i]), j = block_idx(b[i]);
+    Slab& sl = slabs_[s];
+    used_ -= shapes_[sl.shape].block();
+    sl.n_owned--;
+    std::vector<uint64_t> xs;
+    busy(b[i], &xs);
+    xs.push_back(x);
+    sl.st[j] = 2;
+    sl.n_quar++;
+    quarantine_[b[i]] = std::move(xs);
+  }
+}
+
 uint64_t SlabPool::reclaim() {
   uint64_t released = 0;
   std::vector<uint32_t> touched;

@@ -48,6 +48,8 @@ class SlabPool {
   // H1 API.  alloc/free validate everything before changing state (all-or-nothing).
   void alloc(const Shape& sh, int32_t n, aeg_block* out);
   void free(const aeg_block* b, int32_t n);
+  // free, keeping the blocks in the move list until transfer `x` (too) has completed
+  void free_after(const aeg_block* b, int32_t n, uint64_t x);
   uint64_t reclaim();  // release move-list blocks whose transfers all completed
   // Validate that b[0..n) are distinct owned blocks of this pool (and of shape sh if given).
   void check_owned(const aeg_block* b, int32_t n, const Shape* sh, bool distinct = true) const;

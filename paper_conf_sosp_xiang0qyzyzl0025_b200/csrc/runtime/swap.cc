@@ -72,9 +72,8 @@ std::vector<uint64_t> uniq(std::vector<uint64_t> v) {
 
 // Copy-engine DMAs between a staging slot and the host blocks of segment g (layer-major staging
 // image inside the slot).  dir = cudaMemcpyDeviceToHost (swap-out) or HostToDevice (swap-in).
-static void host_dmas(Ctx& c, const Shape& sh, const std::vector<Run>& runs, const Seg& g, char* slot,
-                      cudaMemcpyKind dir, cudaStream_t s) {
-  const SlabPool& hp = c.pool[AEG_POOL_HOST];
+static void host_dmas(const SlabPool& hp, char* hbase, const Shape& sh, const std::vector<Run>& runs, const Seg& g,
+                      char* slot, cudaMemcpyKind dir, cudaStream_t s) {
   const uint64_t Cl = sh.chunk(), hstride = hp.lstride(sh);
   const int32_t nseg = g.i1 - g.i0, nl = g.lb - g.la;
   for (const Run& r : runs) {
@@ -82,7 +81,7 @@ static void host_dmas(Ctx& c, const Shape& sh, const std::vector<Run>& runs, con
     if (a >= b) continue;
     const aeg_block hb = make_block(AEG_POOL_HOST, block_slab(r.first), block_idx(r.first) + uint32_t(a - r.i0));
     const int32_t m = b - a;
-    char* host0 = c.host_kv + hp.off0(hb, sh) + uint64_t(g.la) * hstride;
+    char* host0 = hbase + hp.off0(hb, sh) + uint64_t(g.la) * hstride;
     char* st0 = slot + uint64_t(a - g.i0) * Cl;
     const uint64_t st_pitch = uint64_t(nseg) * Cl;  // next layer inside the slot
     if (hp.layout == AEG_LAYER_MAJOR) {
@@ -165,7 +164,7 @@ uint64_t Ctx::swap_out(const Shape& sh, const aeg_block* dev, const aeg_block* h
     CUDA_TRY(cudaStreamWaitEvent(s_d2h, ring_out.full[slot], 0));
     tr_wait(s_d2h, ring_out.full[slot]);
     if (g.i0 == 0) wait_deps(s_d2h, wdeps, g.la, g.lb);  // rule ❸
-    host_dmas(*this, sh, runs, g, sp, cudaMemcpyDeviceToHost, s_d2h);
+    host_dmas(hp, host_kv, sh, runs, g, sp, cudaMemcpyDeviceToHost, s_d2h);
     if (tracing) tr("op d2h d2h r=SO" + std::to_string(slot) + " w=" + cells(1, hp, host, n, g.la, g.lb, g.i0, g.i1));
     CUDA_TRY(cudaEventRecord(ring_out.free_[slot], s_d2h));
     tr_record(s_d2h, ring_out.free_[slot]);
@@ -183,17 +182,45 @@ uint64_t Ctx::swap_out(const Shape& sh, const aeg_block* dev, const aeg_block* h
 
 // ------------------------------------------------------------------------------ swap-in H4
 uint64_t Ctx::swap_in(const Shape& sh, const aeg_block* host, const aeg_block* dev, int32_t n, uint32_t flags) {
+  return swap_in_from(sh, -1, host, dev, n, 0, flags);
+}
+
+uint64_t Ctx::swap_in_from(const Shape& sh, int32_t peer, const aeg_block* host, const aeg_block* dev, int32_t n,
+                           uint64_t after, uint32_t flags) {
   AEG_REQUIRE(!host_only, AEG_ERR_STATE, "host-only context has no data path");
-  SlabPool &dp = pool[AEG_POOL_DEVICE], &hp = pool[AEG_POOL_HOST];
-  hp.check_owned(host, n, &sh);
+  SlabPool& dp = pool[AEG_POOL_DEVICE];
+  const bool own = peer < 0;
+  SlabPool* hpp = &pool[AEG_POOL_HOST];
+  char* hbase = host_kv;
+  if (own) {
+    hpp->check_owned(host, n, &sh);
+  } else {
+    auto it = peers.find(peer);
+    AEG_REQUIRE(it != peers.end() && it->second->has_host, AEG_ERR_INVALID,
+                "peer %d has no imported shared host region", peer);
+    AEG_REQUIRE(!(flags & AEG_FREE_SRC), AEG_ERR_INVALID, "AEG_FREE_SRC: a peer's host blocks belong to the peer");
+    hpp = &it->second->host_geom;
+    hbase = it->second->host_kv;
+    hpp->check_geometry(host, n, sh);
+    for (int32_t i = 0; i < n; ++i)
+      AEG_REQUIRE(block_pool(host[i]) == AEG_POOL_HOST, AEG_ERR_INVALID, "peer handle is not a host block");
+  }
+  SlabPool& hp = *hpp;
   dp.check_owned(dev, n, &sh);
   AEG_REQUIRE(sh.chunk() <= ring_in.slot_bytes, AEG_ERR_INVALID, "chunk larger than a staging slot");
+  if (after) {
+    auto it = xfers.find(after);
+    AEG_REQUIRE(it == xfers.end() || it->second->L == sh.L || it->second->done_recorded, AEG_ERR_INVALID,
+                "dependency transfer %llu has another layer count", (unsigned long long)after);
+  }
   Xfer* x = new_xfer(X_SWAP_IN, sh.L, false);
   std::vector<uint64_t> rdeps, wdeps;
   if (!(flags & AEG_NO_DEPS)) {
-    for (int32_t i = 0; i < n; ++i) hp.deps_for_read(host[i], rdeps);
+    if (own)
+      for (int32_t i = 0; i < n; ++i) hp.deps_for_read(host[i], rdeps);
     for (int32_t i = 0; i < n; ++i) dp.deps_for_write(dev[i], wdeps);
   }
+  if (after) rdeps.push_back(after);  // rule ❷ across instances (Fig. 10 ③), per layer
   rdeps = uniq(rdeps);
   wdeps = uniq(wdeps);
   char *htab = nullptr, *dtab = nullptr;
@@ -212,7 +239,7 @@ uint64_t Ctx::swap_in(const Shape& sh, const aeg_block* host, const aeg_block* d
     if (g.i0 == 0) wait_deps(s_h2d, rdeps, g.la, g.lb);  // rule ❷ per layer (reading 12)
     CUDA_TRY(cudaStreamWaitEvent(s_h2d, ring_in.free_[slot], 0));
     tr_wait(s_h2d, ring_in.free_[slot]);
-    host_dmas(*this, sh, runs, g, sp, cudaMemcpyHostToDevice, s_h2d);
+    host_dmas(hp, hbase, sh, runs, g, sp, cudaMemcpyHostToDevice, s_h2d);
     if (tracing) tr("op h2d h2d r=" + cells(1, hp, host, n, g.la, g.lb, g.i0, g.i1) + " w=SI" + std::to_string(slot));
     CUDA_TRY(cudaEventRecord(ring_in.full[slot], s_h2d));
     tr_record(s_h2d, ring_in.full[slot]);
@@ -239,9 +266,10 @@ uint64_t Ctx::swap_in(const Shape& sh, const aeg_block* host, const aeg_block* d
   if (n == 0)
     for (int32_t l = 0; l < sh.L; ++l) record(x, l, s_scatter);
   record(x, -1, s_scatter);
-  for (int32_t i = 0; i < n; ++i) hp.note_read(host[i], x->id);
+  if (own)
+    for (int32_t i = 0; i < n; ++i) hp.note_read(host[i], x->id);
   for (int32_t i = 0; i < n; ++i) dp.note_write(dev[i], x->id);
-  if (flags & AEG_FREE_SRC) hp.free(host, n);
+  if (own && (flags & AEG_FREE_SRC)) hp.free(host, n);
   return x->id;
 }
 

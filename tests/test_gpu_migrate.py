@@ -142,3 +142,98 @@ def test_two_process_ipc_migrate():
         if p.is_alive():
             p.kill()
     assert p.exitcode == 0
+
+
+# ------------------------------------------------------------------------------------ NEXT-2
+def _decode_side_host_route(conn):
+    try:
+        _decode_host_route_body(conn)
+    except BaseException:
+        import traceback
+        conn.send(("error", traceback.format_exc()))
+        raise
+
+
+def _decode_host_route_body(conn):
+    """Decode instance of Fig. 10: imports the prefill instance's shared CPU cache and its swap-out
+    events, swaps R1 in from there (C->D) without any host synchronisation on the prefill side's
+    progress, and exports its swap-in so the prefill side can release the CPU blocks."""
+    ctx, dev = make(aeg.LAYER_MAJOR, slab=MIB, nslabs=4)
+    dev.poison(gi.TAG_NEVER)
+    blob_pool, hb, xblob = conn.recv()
+    ctx.import_peer(0, blob_pool)
+    xo = ctx.xfer_import(0, xblob)
+    dc, do = dev.alloc(SH, len(hb))
+    xi = ctx.kv_swap_in_from(SH.as_tuple(), 0, np.array(hb, dtype=np.uint64), dc, after=xo)   # ③④⑤
+    conn.send((ctx.xfer_export(xi), do))
+    for l in range(SH.L):
+        ctx.layer_ready(xi, l, aeg.READY_BLOCK)                                                  # ⑥
+    conn.send(dev.read().tobytes())
+    conn.recv()
+    ctx.shutdown()
+
+
+def test_two_process_host_route_p_c_d():
+    """NEXT-2: prefill P swaps R1 out to its part of the node-shared
+    CPU KV cache (P->C) behind a 0.2 s delay kernel; decode D swaps it in (C->D) waiting only on P's
+    per-layer IPC events (rule ❷); P frees the CPU blocks after importing D's swap-in, so they stay
+    in P's move list until D is done (rule ❸).  D's device image = oracle swap_in∘swap_out."""
+    require_gpu()
+    import torch
+    ctxm = mp.get_context("spawn")
+    parent, child = ctxm.Pipe()
+    p = ctxm.Process(target=_decode_side_host_route, args=(child,))
+    p.start()
+    child.close()
+
+    def recv():
+        assert parent.poll(120), "decode process did not answer"
+        m = parent.recv()
+        if isinstance(m, tuple) and len(m) == 2 and m[0] == "error":
+            raise AssertionError("decode process failed:\n" + m[1])
+        return m
+
+    try:
+        cfg = aeg.default_config(device_kv_bytes=4 * MIB, host_kv_bytes=4 * MIB, dev_slab_bytes=MIB,
+                                 host_slab_bytes=MIB, host_slab_layout=aeg.BLOCK_MAJOR, staging_slot_bytes=MIB,
+                                 staging_slots=2, stage_ring_bytes=4 * MIB, stage_chunk_bytes=MIB,
+                                 table_arena_bytes=2 * MIB, host_threads=1, flags=aeg.CFG_SHARED_HOST)
+        a = aeg.Context(0, cfg)
+        A = Side(a, aeg.POOL_DEVICE, 4 * MIB, MIB, aeg.LAYER_MAJOR)
+        H = Side(a, aeg.POOL_HOST, 4 * MIB, MIB, aeg.BLOCK_MAJOR)
+        A.poison(gi.TAG_NEVER)
+        H.poison(gi.TAG_NEVER)
+        aimg, himg = A.poison_img(gi.TAG_NEVER), H.poison_img(gi.TAG_NEVER)
+        sc, so = A.alloc(SH, 20)
+        fill_blocks(A, aimg, SH, so, [(1, j) for j in range(20)])
+        hc, ho = H.alloc(SH, 20)
+        s = torch.cuda.Stream()
+        from aeg_inputs import dev as Dv
+        Dv.spin(400_000_000, s.cuda_stream)           # the prefill is still running
+        a.stream_fence(s.cuda_stream)
+        xo = a.kv_swap_out(SH.as_tuple(), sc, hc, flags=aeg.FREE_SRC)                            # ①②
+        parent.send((a.export_ipc(), [int(b) for b in hc], a.xfer_export(xo)))
+        xblob, do = recv()
+        xd = a.xfer_import(1, xblob)
+        a.kv_free_after(aeg.POOL_HOST, hc, xd)        # Ry-style: CPU blocks wait in the move list
+        assert a.stats(aeg.POOL_HOST).quarantined_blocks == 20
+        fresh = a.kv_alloc(aeg.POOL_HOST, SH.as_tuple(), 4)      # allocation skips them (❸)
+        assert not {aeg.decode_block(b)[1:] for b in fresh} & set(map(tuple, ho))
+        got = np.frombuffer(recv(), dtype=np.uint8)
+        himg2 = OK.swap_out(aimg, A.geom, himg, H.geom, SH, so, ho)
+        geom = OK.PoolGeom(4 * MIB, MIB, aeg.LAYER_MAJOR)
+        dimg = gi.region_bytes(gi.kv_seed(1), gi.poison_key(gi.TAG_NEVER, 0), geom.nbytes)
+        exp = OK.swap_in(himg2, H.geom, dimg, geom, SH, ho, do)
+        assert first_diff(got, exp) is None
+        for _ in range(2000):                         # step ⑧: reclaimed once D's swap-in completed
+            a.reclaim()
+            if a.stats(aeg.POOL_HOST).quarantined_blocks == 0:
+                break
+        assert a.stats(aeg.POOL_HOST).quarantined_blocks == 0
+        parent.send("bye")
+        a.shutdown()
+    finally:
+        p.join(timeout=30)
+        if p.is_alive():
+            p.kill()
+    assert p.exitcode == 0
