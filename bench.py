@@ -566,7 +566,8 @@ def switch_leg(aeg, torch, n_switch, kernel, descs, mode="staged", caches=None):
                    "h2d_GBps": round(r[0]["bytes_h2d"] / (statistics.median(lat) * 1e6), 1),
                    "eq4_weights_ms_at_64GBps": round(wsize[nm] / (PCIE_NOMINAL * BETA) / 1e6, 1),
                    # N4: Eq. 4 solved for beta on this B200: T = size / (BW * beta)
-                   "eq4_beta_fit": round(wsize[nm] / (PCIE_NOMINAL * 1e9 * statistics.median(lat) / 1e3), 3)}
+                   "eq4_beta_fit": None if mode == "prefetch" else
+                   round(wsize[nm] / (PCIE_NOMINAL * 1e9 * statistics.median(lat) / 1e3), 3)}
     how = {"staged": "weights staged through the 2 GiB pinned Stage Buffer by host threads (3.a)",
            "direct": "weights DMA'd straight from the page-locked Model Cache (registered once)",
            "prefetch": "weights prefetched during the previous turn, relocated on-device at the switch (3.b)"}[mode]

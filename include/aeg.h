@@ -66,7 +66,10 @@ enum {
 enum {
   AEG_FREE_SRC = 1u << 0,  /* free the source blocks once enqueued; they sit in the move list
                               until the transfer completes               */
-  AEG_NO_DEPS = 1u << 1    /* caller guarantees ordering: skip last-writer stream waits (❷❸) */
+  AEG_NO_DEPS = 1u << 1,   /* caller guarantees ordering: skip last-writer stream waits (❷❸) */
+  AEG_IPC_EVENTS = 1u << 2 /* interprocess-capable events, so aeg_xfer_export works across
+                              processes (implied for AEG_CFG_SHARED_HOST contexts, for
+                              aeg_kv_swap_in_from a peer and for migrates to another process)  */
 };
 /* weight split kinds (Megatron-style tensor parallelism, reading 18) */
 enum { AEG_SPLIT_REPLICATED = 0, AEG_SPLIT_COL = 1, AEG_SPLIT_ROW = 2, AEG_SPLIT_VOCAB = 3 };

@@ -114,6 +114,8 @@ static void host_dmas(const SlabPool& hp, char* hbase, const Shape& sh, const st
 // AUTO = BULK (cp.async.bulk through shared memory): measured 5.93 TB/s in-step for the C2 gather vs
 // 5.56 TB/s for LSU with 1 GiB slots (profiles/r01).  Stores into another GPU's pool use LSU under AUTO
 // (plain st.global to peer addresses) unless BULK is requested explicitly.
+#define ipc_events(flags) (((flags) & AEG_IPC_EVENTS) || (cfg.flags & AEG_CFG_SHARED_HOST))
+
 static int impl_of(const aeg_config& cfg) { return cfg.kernel == AEG_KERNEL_LSU ? IMPL_LSU : IMPL_BULK; }
 
 // ----------------------------------------------------------------------------- swap-out H3
@@ -123,7 +125,7 @@ uint64_t Ctx::swap_out(const Shape& sh, const aeg_block* dev, const aeg_block* h
   dp.check_owned(dev, n, &sh);
   hp.check_owned(host, n, &sh);
   AEG_REQUIRE(sh.chunk() <= ring_out.slot_bytes, AEG_ERR_INVALID, "chunk larger than a staging slot");
-  Xfer* x = new_xfer(X_SWAP_OUT, sh.L, false);
+  Xfer* x = new_xfer(X_SWAP_OUT, sh.L, ipc_events(flags));
   std::vector<uint64_t> rdeps, wdeps;
   if (!(flags & AEG_NO_DEPS)) {
     for (int32_t i = 0; i < n; ++i) dp.deps_for_read(dev[i], rdeps);
@@ -213,7 +215,7 @@ uint64_t Ctx::swap_in_from(const Shape& sh, int32_t peer, const aeg_block* host,
     AEG_REQUIRE(it == xfers.end() || it->second->L == sh.L || it->second->done_recorded, AEG_ERR_INVALID,
                 "dependency transfer %llu has another layer count", (unsigned long long)after);
   }
-  Xfer* x = new_xfer(X_SWAP_IN, sh.L, false);
+  Xfer* x = new_xfer(X_SWAP_IN, sh.L, ipc_events(flags) || !own);
   std::vector<uint64_t> rdeps, wdeps;
   if (!(flags & AEG_NO_DEPS)) {
     if (own)
@@ -297,7 +299,7 @@ uint64_t Ctx::migrate(const Shape& sh, const aeg_block* src, int32_t peer, const
     dg = &P->geom;
     dbase = P->dev_kv;
   }
-  Xfer* x = new_xfer(X_MIGRATE, sh.L, peer >= 0 && !P->same_process);
+  Xfer* x = new_xfer(X_MIGRATE, sh.L, ipc_events(flags) || (peer >= 0 && !P->same_process));
   std::vector<uint64_t> rdeps, wdeps;
   if (!(flags & AEG_NO_DEPS)) {
     for (int32_t i = 0; i < n; ++i) dp.deps_for_read(src[i], rdeps);

@@ -144,7 +144,18 @@ struct WeightPipe {
       if (v != ~0ull) v -= 1;  // index of the last byte
     try {
       if (j->direct) {
+        // Pace the issue: at most kWindow chunks of DMA queued on s_weights, so copies other
+        // streams enqueue meanwhile (the switch's KV swap-in) are not stuck behind the whole model.
+        constexpr int kWindow = 4;
+        uint64_t since = 0, marks = 0;
         for (size_t k = 0; k < j->d.size(); ++k) {
+          if (since >= chunk) {
+            const int slot = int(marks++ % uint64_t(kWindow));
+            if (marks > uint64_t(kWindow)) CUDA_TRY(cudaEventSynchronize(slot_ev[slot]));
+            CUDA_TRY(cudaEventRecord(slot_ev[slot], s));
+            since = 0;
+          }
+          since += j->size[k];
           const aeg_weight_desc& d = j->d[k];
           char* dst = c->dev_w + j->off[k];
           const char* src = static_cast<const char*>(d.host_src);
