@@ -45,6 +45,21 @@ void set_device(Ctx& c) {
   if (!c.host_only) CUDA_TRY(cudaSetDevice(c.device));
 }
 
+// Run one data-path enqueue; if it throws after its transfer was created, drain and mark it failed
+// (Ctx::abort_enqueue) so no reader can block on an event that will never be recorded.
+template <class F>
+uint64_t enqueue(Ctx& c, F&& f) {
+  c.enqueuing = nullptr;
+  try {
+    const uint64_t x = f();
+    c.enqueuing = nullptr;
+    return x;
+  } catch (...) {
+    c.abort_enqueue();
+    throw;
+  }
+}
+
 constexpr uint32_t kIpcMagic = 0xAE6A1BC1u, kXferMagic = 0xAE6A1BC2u;
 
 struct IpcBlob {
@@ -228,7 +243,7 @@ int aeg_kv_swap_out(aeg_ctx ctx, const aeg_kv_shape* shape, const aeg_block* dev
     const aeg::Shape sh = aeg::Shape::from(shape);
     std::lock_guard<std::mutex> g(c.mu);
     set_device(c);
-    *out = c.swap_out(sh, dev, host, n, flags);
+    *out = enqueue(c, [&] { return c.swap_out(sh, dev, host, n, flags); });
     return AEG_OK;
   });
 }
@@ -241,7 +256,7 @@ int aeg_kv_swap_in(aeg_ctx ctx, const aeg_kv_shape* shape, const aeg_block* host
     const aeg::Shape sh = aeg::Shape::from(shape);
     std::lock_guard<std::mutex> g(c.mu);
     set_device(c);
-    *out = c.swap_in(sh, host, dev, n, flags);
+    *out = enqueue(c, [&] { return c.swap_in(sh, host, dev, n, flags); });
     return AEG_OK;
   });
 }
@@ -254,7 +269,7 @@ int aeg_kv_migrate(aeg_ctx ctx, const aeg_kv_shape* shape, const aeg_block* src,
     const aeg::Shape sh = aeg::Shape::from(shape);
     std::lock_guard<std::mutex> g(c.mu);
     set_device(c);
-    *out = c.migrate(sh, src, peer, dst, n, flags);
+    *out = enqueue(c, [&] { return c.migrate(sh, src, peer, dst, n, flags); });
     return AEG_OK;
   });
 }
@@ -267,7 +282,7 @@ int aeg_kv_swap_in_from(aeg_ctx ctx, const aeg_kv_shape* shape, int32_t peer, co
     const aeg::Shape sh = aeg::Shape::from(shape);
     std::lock_guard<std::mutex> g(c.mu);
     set_device(c);
-    *out = c.swap_in_from(sh, peer, peer_host, dev, n, after, flags);
+    *out = enqueue(c, [&] { return c.swap_in_from(sh, peer, peer_host, dev, n, after, flags); });
     return AEG_OK;
   });
 }
@@ -369,7 +384,7 @@ int aeg_weights_relocate(aeg_ctx ctx, uint64_t src_off, uint64_t dst_off, uint64
     set_device(c);
     // rule ❷: the prefetched bytes must have been issued on s_weights before the move
     c.cv.wait(g, [&] { return c.w_inflight == 0; });
-    *out = c.relocate(src_off, dst_off, bytes);
+    *out = enqueue(c, [&] { return c.relocate(src_off, dst_off, bytes); });
     return AEG_OK;
   });
 }

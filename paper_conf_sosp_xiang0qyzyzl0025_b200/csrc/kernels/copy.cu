@@ -11,6 +11,7 @@
 // Both are persistent: the grid is one wave (148 SMs x resident CTAs) striding over items.
 #include <cuda_runtime.h>
 
+#include <atomic>
 #include <cstdint>
 
 #include "copy.h"
@@ -183,11 +184,15 @@ cudaError_t launch_t(const CopyArgs& a, int impl, int max_ctas, cudaStream_t s) 
   const uint64_t items_lsu = uint64_t(a.nl) * a.n * ((a.chunk + kLsuPiece - 1) / kLsuPiece);
   if (items_lsu == 0) return cudaSuccess;
   if (impl == IMPL_BULK) {
-    static bool attr = false;
-    if (!attr) {
-      cudaError_t e = cudaFuncSetAttribute(copy_bulk<SP, DP>, cudaFuncAttributeMaxDynamicSharedMemorySize, kBulkSmem);
+    static std::atomic<uint64_t> attr_set{0};  // per-device bit: opt-in smem attribute applied
+    int dev = 0;
+    cudaError_t e = cudaGetDevice(&dev);
+    if (e != cudaSuccess) return e;
+    const uint64_t bit = 1ull << (dev & 63);
+    if (!(attr_set.load() & bit)) {
+      e = cudaFuncSetAttribute(copy_bulk<SP, DP>, cudaFuncAttributeMaxDynamicSharedMemorySize, kBulkSmem);
       if (e != cudaSuccess) return e;
-      attr = true;
+      attr_set.fetch_or(bit);
     }
     const uint64_t items = uint64_t(a.nl) * a.n * ((a.chunk + kBulkPiece - 1) / kBulkPiece);
     uint64_t grid = max_ctas > 0 ? uint64_t(max_ctas) : uint64_t(kSMs);

@@ -284,7 +284,6 @@ void Ctx::housekeeping() {
       ++it;
     }
   }
-  static int sweep = 0;
   if (++sweep % 64 == 0) {
     pool[0].forget_completed();
     pool[1].forget_completed();
@@ -321,7 +320,25 @@ Xfer* Ctx::new_xfer(int kind, int32_t L, bool ipc) {
   }
   Xfer* raw = x.get();
   xfers.emplace(raw->id, std::move(x));
+  enqueuing = raw;
   return raw;
+}
+
+// A CUDA error interrupted an enqueue: some of the transfer's work may be queued, some not, and
+// some events never recorded.  Drain the library streams (error path only), then mark every layer
+// recorded + the transfer complete and failed, so no waiter blocks and readiness reports the error.
+void Ctx::abort_enqueue() {
+  Xfer* x = enqueuing;
+  enqueuing = nullptr;
+  if (!x || host_only) return;
+  for (cudaStream_t s : {s_gather, s_d2h, s_h2d, s_scatter, s_migrate}) cudaStreamSynchronize(s);
+  (void)cudaGetLastError();
+  std::fill(x->recorded.begin(), x->recorded.end(), uint8_t(1));
+  x->done_recorded = true;
+  x->failed = true;
+  x->released = true;  // the caller never received its id: reap it
+  x->complete.store(true);
+  cv.notify_all();
 }
 
 Xfer* Ctx::get_xfer(uint64_t id) {
@@ -372,6 +389,7 @@ int Ctx::layer_ready(uint64_t id, int32_t layer, int mode, cudaStream_t s) {
     AEG_REQUIRE(mode == AEG_READY_QUERY, AEG_ERR_STATE, "host-only context: QUERY only");
     return x->complete.load() ? AEG_OK : AEG_NOT_READY;
   }
+  AEG_REQUIRE(!x->failed, AEG_ERR_CUDA, "transfer %llu failed while being enqueued", (unsigned long long)id);
   auto recorded = [&] { return layer < 0 ? x->done_recorded : x->recorded[layer] != 0; };
   if (!recorded()) {
     if (mode == AEG_READY_QUERY) return AEG_NOT_READY;

@@ -45,6 +45,7 @@ struct Xfer {
   std::atomic<bool> complete{false};
   bool released = false;
   bool owns_events = true;          // imported transfers borrow cached peer events
+  bool failed = false;              // enqueue was interrupted by an error (events force-recorded)
   bool debug_done = false;          // host-only synthetic transfers
   uint64_t table_mark = 0;          // table-arena end offset to release on completion
 };
@@ -134,6 +135,7 @@ struct Ctx {
 
   std::thread daemon;
   bool stop = false;
+  int sweep = 0;  // housekeeping rounds (access-map pruning cadence)
   std::unique_ptr<WeightPipe> wp;
   std::unordered_map<int, std::unique_ptr<Peer>> peers;
   std::vector<std::pair<char*, uint64_t>> registered;
@@ -158,6 +160,8 @@ struct Ctx {
   void poll();                     // query events of in-flight transfers (caller holds mu)
   void housekeeping();             // poll + reclaim + release tables + reap (caller holds mu)
   Xfer* new_xfer(int kind, int32_t L, bool ipc);
+  Xfer* enqueuing = nullptr;       // transfer whose enqueue is in progress (error recovery)
+  void abort_enqueue();            // error path: drain library streams, mark the transfer failed
   Xfer* get_xfer(uint64_t id);     // STATE if unknown/released
   cudaEvent_t take_event(bool ipc);
   void give_event(cudaEvent_t e, bool ipc);

@@ -219,7 +219,13 @@ struct WeightPipe {
       c->w_inflight--;
     } catch (const Error& e) {
       fprintf(stderr, "aegkv: weight pipeline failed: %s\n", e.what());
+      cudaStreamSynchronize(s);
+      (void)cudaGetLastError();
       std::lock_guard<std::mutex> g(c->mu);
+      std::fill(j->x->recorded.begin(), j->x->recorded.end(), uint8_t(1));  // never block a waiter
+      j->x->done_recorded = true;
+      j->x->failed = true;
+      j->x->complete.store(true);
       c->w_inflight--;
     }
     c->cv.notify_all();

@@ -160,6 +160,7 @@ def _decode_host_route_body(conn):
     progress, and exports its swap-in so the prefill side can release the CPU blocks."""
     ctx, dev = make(aeg.LAYER_MAJOR, slab=MIB, nslabs=4)
     dev.poison(gi.TAG_NEVER)
+    conn.send("ready")
     blob_pool, hb, xblob = conn.recv()
     ctx.import_peer(0, blob_pool)
     xo = ctx.xfer_import(0, xblob)
@@ -207,9 +208,10 @@ def test_two_process_host_route_p_c_d():
         sc, so = A.alloc(SH, 20)
         fill_blocks(A, aimg, SH, so, [(1, j) for j in range(20)])
         hc, ho = H.alloc(SH, 20)
+        assert recv() == "ready"                      # the decode instance is up
         s = torch.cuda.Stream()
         from aeg_inputs import dev as Dv
-        Dv.spin(400_000_000, s.cuda_stream)           # the prefill is still running
+        Dv.spin(1_000_000_000, s.cuda_stream)         # the prefill is still running (~0.5 s)
         a.stream_fence(s.cuda_stream)
         xo = a.kv_swap_out(SH.as_tuple(), sc, hc, flags=aeg.FREE_SRC)                            # ①②
         parent.send((a.export_ipc(), [int(b) for b in hc], a.xfer_export(xo)))
