@@ -165,13 +165,7 @@ void Ctx::init(int dev, const aeg_config& c) {
   CUDA_TRY(cudaEventCreateWithFlags(&fence_ev, cudaEventDisableTiming));
   for (Ring* r : {&ring_out, &ring_in}) {
     r->slot_bytes = cfg.staging_slot_bytes;
-    r->n = cfg.staging_slots;
-    r->full.resize(r->n);
-    r->free_.resize(r->n);
-    for (int i = 0; i < r->n; ++i) {
-      CUDA_TRY(cudaEventCreateWithFlags(&r->full[i], cudaEventDisableTiming));
-      CUDA_TRY(cudaEventCreateWithFlags(&r->free_[i], cudaEventDisableTiming));
-    }
+    r->bytes = cfg.staging_slot_bytes * uint64_t(cfg.staging_slots);
   }
   weights_start();
   if (!(cfg.flags & AEG_CFG_NO_DAEMON)) daemon = std::thread([this] { daemon_loop(); });
@@ -205,10 +199,8 @@ void Ctx::shutdown() {
     cudaEventDestroy(t.a);
     cudaEventDestroy(t.b);
   }
-  for (Ring* r : {&ring_out, &ring_in}) {
-    for (cudaEvent_t e : r->full) cudaEventDestroy(e);
-    for (cudaEvent_t e : r->free_) cudaEventDestroy(e);
-  }
+  ring_out.destroy();
+  ring_in.destroy();
   for (auto& kv : peers) {
     Peer* p = kv.second.get();
     for (auto& e : p->events) cudaEventDestroy(e.second);
@@ -225,6 +217,52 @@ void Ctx::shutdown() {
     if (s) cudaStreamDestroy(s);
   if (dev_mem) cudaFree(dev_mem);
   if (host_mem) unpin_host(host_mem, host_mem_bytes);
+}
+
+// --------------------------------------------------------------------------- staging ring
+char* Ring::acquire(uint64_t size, cudaStream_t producer, cudaEvent_t* full, cudaEvent_t* freed, uint64_t* off,
+                   std::vector<cudaEvent_t>* waited) {
+  AEG_REQUIRE(size > 0 && size <= slot_bytes, AEG_ERR_INVALID, "staging segment of %llu bytes exceeds a slot",
+              (unsigned long long)size);
+  const uint64_t pos = head % bytes;
+  if (pos + size > bytes) head += bytes - pos;  // never wrap inside a segment
+  const uint64_t start = head, end = head + size;
+  // every older segment that started before end - bytes shares bytes with [start, end)
+  while (!live.empty() && end > bytes && live.front().start < end - bytes) {
+    Seg& s = live.front();
+    CUDA_TRY(cudaStreamWaitEvent(producer, s.freed, 0));
+    if (waited) waited->push_back(s.freed);
+    pool.push_back(s.full);   // both events were already waited on; safe to re-record
+    pool.push_back(s.freed);
+    live.pop_front();
+  }
+  auto take = [&]() {
+    if (!pool.empty()) {
+      cudaEvent_t e = pool.back();
+      pool.pop_back();
+      return e;
+    }
+    cudaEvent_t e;
+    CUDA_TRY(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
+    return e;
+  };
+  Seg s{start, end, take(), take()};
+  live.push_back(s);
+  head = end;
+  *full = s.full;
+  *freed = s.freed;
+  *off = start % bytes;
+  return base + start % bytes;
+}
+
+void Ring::destroy() {
+  for (auto& s : live) {
+    cudaEventDestroy(s.full);
+    cudaEventDestroy(s.freed);
+  }
+  for (cudaEvent_t e : pool) cudaEventDestroy(e);
+  live.clear();
+  pool.clear();
 }
 
 // ------------------------------------------------------------------------------- daemon ⑧

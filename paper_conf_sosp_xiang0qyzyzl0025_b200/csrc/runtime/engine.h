@@ -50,16 +50,28 @@ struct Xfer {
   uint64_t table_mark = 0;          // table-arena end offset to release on completion
 };
 
-// Ring of device staging slots for one direction of KV swaps.  Slot reuse is ordered entirely
-// on the GPU: the producer stream waits on free[slot] (recorded by the consumer after it used
-// the slot) and the consumer waits on full[slot] (rule ❸ at ring level, no host blocking).
+// Device staging ring for one direction of KV swaps: a byte ring (slots x slot_bytes) in which
+// segments of any size <= slot_bytes are packed back to back.  Reuse is ordered entirely on the
+// GPU (rule ❸ at ring level, no host blocking): a new segment's producer stream waits on the
+// `freed` events of the older segments whose bytes it overwrites; its consumer waits on `full`.
+// Packing matters because one copy engine serves all H2D streams FIFO (profiles/r01/ce_probe.txt):
+// a transfer of many small segments must be enqueued at once, not trickle in as fixed slots free up.
 struct Ring {
+  struct Seg {
+    uint64_t start, end;  // monotonic byte positions
+    cudaEvent_t full, freed;
+  };
   char* base = nullptr;
-  uint64_t slot_bytes = 0;
-  int n = 0;
-  uint64_t next = 0;
-  std::vector<cudaEvent_t> full, free_;
-  char* slot(int i) const { return base + uint64_t(i) * slot_bytes; }
+  uint64_t slot_bytes = 0;  // max segment size
+  uint64_t bytes = 0;       // ring size
+  uint64_t head = 0;        // monotonic
+  std::deque<Seg> live;
+  std::vector<cudaEvent_t> pool;
+  // Reserve `size` bytes; makes `producer` wait for the segments being overwritten.  Returns the
+  // device pointer and the segment's (full, freed) events.
+  char* acquire(uint64_t size, cudaStream_t producer, cudaEvent_t* full, cudaEvent_t* freed, uint64_t* off,
+                std::vector<cudaEvent_t>* waited);
+  void destroy();
 };
 
 // Device block-table arena (+ pinned host mirror), allocated FIFO per transfer and released when

@@ -62,6 +62,18 @@ std::vector<Run> runs_of(const aeg_block* h, int32_t n) {
   return r;
 }
 
+// Trace cells of a staging-ring range (16 KiB granules), so the rule checker sees ring reuse.
+std::string ring_cells(const char* tag, uint64_t off, uint64_t size) {
+  std::string s;
+  for (uint64_t g = off >> 14; g < (off + size + (1u << 14) - 1) >> 14; ++g) {
+    if (!s.empty()) s += ',';
+    s += tag;
+    s += ':';
+    s += std::to_string(g);
+  }
+  return s;
+}
+
 std::vector<uint64_t> uniq(std::vector<uint64_t> v) {
   std::sort(v.begin(), v.end());
   v.erase(std::unique(v.begin(), v.end()), v.end());
@@ -144,11 +156,13 @@ uint64_t Ctx::swap_out(const Shape& sh, const aeg_block* dev, const aeg_block* h
   const auto runs = runs_of(host, n);
   const uint64_t dstride = dp.lstride(sh);
   for (const Seg& g : segs) {
-    const int slot = int(ring_out.next++ % uint64_t(ring_out.n));
-    char* sp = ring_out.slot(slot);
     if (g.i0 == 0) wait_deps(s_gather, rdeps, g.la, g.lb);  // rule ❷
-    CUDA_TRY(cudaStreamWaitEvent(s_gather, ring_out.free_[slot], 0));
-    tr_wait(s_gather, ring_out.free_[slot]);
+    cudaEvent_t full, freed;
+    uint64_t roff;
+    std::vector<cudaEvent_t> waited;
+    const uint64_t seg_bytes = uint64_t(g.lb - g.la) * uint64_t(g.i1 - g.i0) * sh.chunk();
+    char* sp = ring_out.acquire(seg_bytes, s_gather, &full, &freed, &roff, tracing ? &waited : nullptr);
+    for (cudaEvent_t e : waited) tr_wait(s_gather, e);
     CopyArgs a;
     a.src = dev_kv;
     a.src_off = reinterpret_cast<const uint64_t*>(dtab) + g.i0;
@@ -159,17 +173,19 @@ uint64_t Ctx::swap_out(const Shape& sh, const aeg_block* dev, const aeg_block* h
     a.nl = g.lb - g.la;
     a.n = g.i1 - g.i0;
     launch(0, a, s_gather, impl_of(cfg), 0);
-    if (tracing) tr("op gather gather r=" + cells(0, dp, dev, n, g.la, g.lb, g.i0, g.i1) + " w=SO" + std::to_string(slot));
-    CUDA_TRY(cudaEventRecord(ring_out.full[slot], s_gather));
-    tr_record(s_gather, ring_out.full[slot]);
+    if (tracing)
+      tr("op gather gather r=" + cells(0, dp, dev, n, g.la, g.lb, g.i0, g.i1) + " w=" + ring_cells("SO", roff, seg_bytes));
+    CUDA_TRY(cudaEventRecord(full, s_gather));
+    tr_record(s_gather, full);
 
-    CUDA_TRY(cudaStreamWaitEvent(s_d2h, ring_out.full[slot], 0));
-    tr_wait(s_d2h, ring_out.full[slot]);
+    CUDA_TRY(cudaStreamWaitEvent(s_d2h, full, 0));
+    tr_wait(s_d2h, full);
     if (g.i0 == 0) wait_deps(s_d2h, wdeps, g.la, g.lb);  // rule ❸
     host_dmas(hp, host_kv, sh, runs, g, sp, cudaMemcpyDeviceToHost, s_d2h);
-    if (tracing) tr("op d2h d2h r=SO" + std::to_string(slot) + " w=" + cells(1, hp, host, n, g.la, g.lb, g.i0, g.i1));
-    CUDA_TRY(cudaEventRecord(ring_out.free_[slot], s_d2h));
-    tr_record(s_d2h, ring_out.free_[slot]);
+    if (tracing)
+      tr("op d2h d2h r=" + ring_cells("SO", roff, seg_bytes) + " w=" + cells(1, hp, host, n, g.la, g.lb, g.i0, g.i1));
+    CUDA_TRY(cudaEventRecord(freed, s_d2h));
+    tr_record(s_d2h, freed);
     if (g.i1 == n)
       for (int32_t l = g.la; l < g.lb; ++l) record(x, l, s_d2h);
   }
@@ -236,18 +252,21 @@ uint64_t Ctx::swap_in_from(const Shape& sh, int32_t peer, const aeg_block* host,
   const auto runs = runs_of(host, n);
   const uint64_t dstride = dp.lstride(sh);
   for (const Seg& g : segs) {
-    const int slot = int(ring_in.next++ % uint64_t(ring_in.n));
-    char* sp = ring_in.slot(slot);
     if (g.i0 == 0) wait_deps(s_h2d, rdeps, g.la, g.lb);  // rule ❷ per layer (reading 12)
-    CUDA_TRY(cudaStreamWaitEvent(s_h2d, ring_in.free_[slot], 0));
-    tr_wait(s_h2d, ring_in.free_[slot]);
+    cudaEvent_t full, freed;
+    uint64_t roff;
+    std::vector<cudaEvent_t> waited;
+    const uint64_t seg_bytes = uint64_t(g.lb - g.la) * uint64_t(g.i1 - g.i0) * sh.chunk();
+    char* sp = ring_in.acquire(seg_bytes, s_h2d, &full, &freed, &roff, tracing ? &waited : nullptr);
+    for (cudaEvent_t e : waited) tr_wait(s_h2d, e);
     host_dmas(hp, hbase, sh, runs, g, sp, cudaMemcpyHostToDevice, s_h2d);
-    if (tracing) tr("op h2d h2d r=" + cells(1, hp, host, n, g.la, g.lb, g.i0, g.i1) + " w=SI" + std::to_string(slot));
-    CUDA_TRY(cudaEventRecord(ring_in.full[slot], s_h2d));
-    tr_record(s_h2d, ring_in.full[slot]);
+    if (tracing)
+      tr("op h2d h2d r=" + cells(1, hp, host, n, g.la, g.lb, g.i0, g.i1) + " w=" + ring_cells("SI", roff, seg_bytes));
+    CUDA_TRY(cudaEventRecord(full, s_h2d));
+    tr_record(s_h2d, full);
 
-    CUDA_TRY(cudaStreamWaitEvent(s_scatter, ring_in.full[slot], 0));
-    tr_wait(s_scatter, ring_in.full[slot]);
+    CUDA_TRY(cudaStreamWaitEvent(s_scatter, full, 0));
+    tr_wait(s_scatter, full);
     if (g.i0 == 0) wait_deps(s_scatter, wdeps, g.la, g.lb);  // rule ❸
     CopyArgs a;
     a.src = sp;
@@ -259,9 +278,10 @@ uint64_t Ctx::swap_in_from(const Shape& sh, int32_t peer, const aeg_block* host,
     a.nl = g.lb - g.la;
     a.n = g.i1 - g.i0;
     launch(1, a, s_scatter, impl_of(cfg), 0);
-    if (tracing) tr("op scatter scatter r=SI" + std::to_string(slot) + " w=" + cells(0, dp, dev, n, g.la, g.lb, g.i0, g.i1));
-    CUDA_TRY(cudaEventRecord(ring_in.free_[slot], s_scatter));
-    tr_record(s_scatter, ring_in.free_[slot]);
+    if (tracing)
+      tr("op scatter scatter r=" + ring_cells("SI", roff, seg_bytes) + " w=" + cells(0, dp, dev, n, g.la, g.lb, g.i0, g.i1));
+    CUDA_TRY(cudaEventRecord(freed, s_scatter));
+    tr_record(s_scatter, freed);
     if (g.i1 == n)
       for (int32_t l = g.la; l < g.lb; ++l) record(x, l, s_scatter);
   }

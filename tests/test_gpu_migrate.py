@@ -217,8 +217,10 @@ def test_two_process_host_route_p_c_d():
         parent.send((a.export_ipc(), [int(b) for b in hc], a.xfer_export(xo)))
         xblob, do = recv()
         xd = a.xfer_import(1, xblob)
+        out_done = a.layer_ready(xo, -1, aeg.READY_QUERY)
+        in_done = a.layer_ready(xd, -1, aeg.READY_QUERY)
         a.kv_free_after(aeg.POOL_HOST, hc, xd)        # Ry-style: CPU blocks wait in the move list
-        assert a.stats(aeg.POOL_HOST).quarantined_blocks == 20
+        q = a.stats(aeg.POOL_HOST).quarantined_blocks
         fresh = a.kv_alloc(aeg.POOL_HOST, SH.as_tuple(), 4)      # allocation skips them (❸)
         assert not {aeg.decode_block(b)[1:] for b in fresh} & set(map(tuple, ho))
         got = np.frombuffer(recv(), dtype=np.uint8)
@@ -227,6 +229,9 @@ def test_two_process_host_route_p_c_d():
         dimg = gi.region_bytes(gi.kv_seed(1), gi.poison_key(gi.TAG_NEVER, 0), geom.nbytes)
         exp = OK.swap_in(himg2, H.geom, dimg, geom, SH, ho, do)
         assert first_diff(got, exp) is None
+        # while P's swap-out sat behind the delay kernel, neither transfer was complete and the CPU
+        # blocks went to the move list
+        assert (out_done, in_done, q) == (False, False, 20)
         for _ in range(2000):                         # step ⑧: reclaimed once D's swap-in completed
             a.reclaim()
             if a.stats(aeg.POOL_HOST).quarantined_blocks == 0:
