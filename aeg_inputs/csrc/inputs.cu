@@ -91,6 +91,12 @@ __global__ void consume_chunks(const char* base, const uint64_t* off, uint64_t n
   if ((threadIdx.x & 31) == 0 && acc) atomicXor(out, (unsigned long long)acc);
 }
 
+// Deterministic race-test gate: holds its stream until the host writes a nonzero value into the
+// pinned (device-mapped) flag.
+__global__ void gate(const volatile int* flag) {
+  while (*flag == 0) __nanosleep(1000);
+}
+
 __global__ void spin(long long cycles) {
   const long long t0 = clock64();
   while (clock64() - t0 < cycles) {
@@ -206,6 +212,11 @@ int aegin_consume(const void* base, const uint64_t* dev_off, uint64_t n, uint64_
 int aegin_copy(void* dst, const void* src, uint64_t n) { return int(cudaMemcpy(dst, src, n, cudaMemcpyDefault)); }
 
 int aegin_sync(void) { return int(cudaDeviceSynchronize()); }
+
+int aegin_gate(const void* pinned_flag, void* stream) {
+  gate<<<1, 1, 0, static_cast<cudaStream_t>(stream)>>>(static_cast<const volatile int*>(pinned_flag));
+  return int(cudaGetLastError());
+}
 
 int aegin_spin(long long cycles, void* stream) {
   spin<<<1, 1, 0, static_cast<cudaStream_t>(stream)>>>(cycles);

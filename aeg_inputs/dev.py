@@ -27,6 +27,7 @@ def lib():
             "aegin_verify_region": [P, U64, U64, U64, PU64, PU64, P],
             "aegin_consume": [P, P, U64, U64, P, P],
             "aegin_spin": [C.c_longlong, P],
+            "aegin_gate": [P, P],
             "aegin_copy": [P, P, U64],
             "aegin_sync": [],
             "aegin_host_fill": [P, U64, U64, U64, C.c_int],
@@ -77,6 +78,21 @@ def consume(base: int, dev_offsets_ptr: int, n: int, chunk: int, out_ptr: int, s
 
 def spin(cycles: int, stream: int = 0):
     _ck(lib().aegin_spin(int(cycles), P(stream)))
+
+
+class Gate:
+    """Holds a stream until open(): a kernel polling a pinned host flag (deterministic race tests)."""
+
+    def __init__(self):
+        import torch
+        self.flag = torch.zeros(1, dtype=torch.int32, pin_memory=True)
+
+    def close_on(self, stream: int):
+        self.flag[0] = 0
+        _ck(lib().aegin_gate(P(self.flag.data_ptr()), P(stream)))
+
+    def open(self):
+        self.flag[0] = 1
 
 
 def copy(dst: int, src: int, nbytes: int):

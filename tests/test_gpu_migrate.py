@@ -211,7 +211,8 @@ def test_two_process_host_route_p_c_d():
         assert recv() == "ready"                      # the decode instance is up
         s = torch.cuda.Stream()
         from aeg_inputs import dev as Dv
-        Dv.spin(1_000_000_000, s.cuda_stream)         # the prefill is still running (~0.5 s)
+        gate = Dv.Gate()
+        gate.close_on(s.cuda_stream)                  # the prefill is still running until gate.open()
         a.stream_fence(s.cuda_stream)
         xo = a.kv_swap_out(SH.as_tuple(), sc, hc, flags=aeg.FREE_SRC)                            # ①②
         parent.send((a.export_ipc(), [int(b) for b in hc], a.xfer_export(xo)))
@@ -222,16 +223,15 @@ def test_two_process_host_route_p_c_d():
         a.kv_free_after(aeg.POOL_HOST, hc, xd)        # Ry-style: CPU blocks wait in the move list
         q = a.stats(aeg.POOL_HOST).quarantined_blocks
         fresh = a.kv_alloc(aeg.POOL_HOST, SH.as_tuple(), 4)      # allocation skips them (❸)
+        assert (out_done, in_done, q) == (False, False, 20)
         assert not {aeg.decode_block(b)[1:] for b in fresh} & set(map(tuple, ho))
+        gate.open()                                   # prefill done: P->C runs, then C->D on D's side
         got = np.frombuffer(recv(), dtype=np.uint8)
         himg2 = OK.swap_out(aimg, A.geom, himg, H.geom, SH, so, ho)
         geom = OK.PoolGeom(4 * MIB, MIB, aeg.LAYER_MAJOR)
         dimg = gi.region_bytes(gi.kv_seed(1), gi.poison_key(gi.TAG_NEVER, 0), geom.nbytes)
         exp = OK.swap_in(himg2, H.geom, dimg, geom, SH, ho, do)
         assert first_diff(got, exp) is None
-        # while P's swap-out sat behind the delay kernel, neither transfer was complete and the CPU
-        # blocks went to the move list
-        assert (out_done, in_done, q) == (False, False, 20)
         for _ in range(2000):                         # step ⑧: reclaimed once D's swap-in completed
             a.reclaim()
             if a.stats(aeg.POOL_HOST).quarantined_blocks == 0:

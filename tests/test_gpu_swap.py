@@ -117,7 +117,8 @@ def test_c1_swap_in_chained_on_swap_out_without_host_sync():
         dc, do = requests(dev, dimg, SH)
         hc, ho = host.alloc(SH, len(do))
         s = torch.cuda.Stream()
-        D.spin(200_000_000, s.cuda_stream)            # ~0.1 s at 2 GHz
+        gate = D.Gate()
+        gate.close_on(s.cuda_stream)                  # the "prefill" runs until gate.open()
         ctx.stream_fence(s.cuda_stream)               # swap-out ordered after the "prefill"
         ctx.trace_enable(True)
         x = ctx.kv_swap_out(SH.as_tuple(), dc, hc, flags=aeg.FREE_SRC)
@@ -126,7 +127,9 @@ def test_c1_swap_in_chained_on_swap_out_without_host_sync():
         xo = dev.oracle.begin(do)
         dev.oracle.free(do)
         y = ctx.kv_swap_in(SH.as_tuple(), hc, nc)
-        assert not ctx.layer_ready(x, 0, aeg.READY_QUERY)   # still held back by the spin kernel
+        assert not ctx.layer_ready(x, 0, aeg.READY_QUERY)   # still held back by the gate
+        assert not ctx.layer_ready(y, 0, aeg.READY_QUERY)   # rule ❷: the swap-in waits for it
+        gate.open()
         himg = OK.swap_out(dimg, dev.geom, himg, host.geom, SH, do, ho)
         exp = OK.swap_in(himg, host.geom, dimg, dev.geom, SH, ho, no)
         cons = torch.cuda.Stream()
