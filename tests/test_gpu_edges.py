@@ -1,0 +1,144 @@
+"""GPU edge cases of the ABI: empty transfers, a one-layer shape, ragged single blocks, a block larger
+than a staging slot, shapes whose chunk is not 16-byte aligned, OOM without state change, readiness
+of released / unknown transfers — each against the oracle or the documented error code."""
+import numpy as np
+import pytest
+
+import aeg_inputs as gi
+import paper_conf_sosp_xiang0qyzyzl0025_b200 as aeg
+from oracle import kv as OK
+from oracle.shape import KVShape
+
+from .gpu_harness import Side, fill_blocks, first_diff, require_gpu
+
+pytestmark = pytest.mark.gpu
+MIB = 1 << 20
+
+
+def make(slot=MIB, dev_slabs=4, host_slabs=4, slab=MIB):
+    cfg = aeg.default_config(device_kv_bytes=dev_slabs * slab, host_kv_bytes=host_slabs * slab, dev_slab_bytes=slab,
+                             host_slab_bytes=slab, staging_slot_bytes=slot, staging_slots=2,
+                             stage_ring_bytes=4 * MIB, stage_chunk_bytes=MIB, table_arena_bytes=2 * MIB,
+                             host_threads=1)
+    ctx = aeg.Context(0, cfg)
+    return ctx, Side(ctx, 0, dev_slabs * slab, slab, 0), Side(ctx, 1, host_slabs * slab, slab, 0)
+
+
+def test_empty_transfers_are_ready():
+    require_gpu()
+    ctx, _, _ = make()
+    try:
+        sh = (2, 1, 64, 2, 16)
+        for x in (ctx.kv_swap_out(sh, [], []), ctx.kv_swap_in(sh, [], []), ctx.kv_migrate(sh, [], -1, [])):
+            ctx.layer_ready(x, -1, aeg.READY_BLOCK)
+            assert all(ctx.layer_ready(x, l, aeg.READY_QUERY) for l in range(2))
+            ctx.xfer_release(x)
+    finally:
+        ctx.shutdown()
+
+
+@pytest.mark.parametrize("shape", [(1, 1, 8, 2, 1), (3, 1, 8, 2, 1), (1, 2, 64, 2, 16)])
+def test_small_shapes_round_trip(shape):
+    """One-layer shapes and 1-token blocks (chunk = 32 B): ragged, launch-bound, still bit-exact."""
+    require_gpu()
+    sh = KVShape(*shape)
+    ctx, dev, host = make()
+    try:
+        dev.poison(gi.TAG_NEVER)
+        host.poison(gi.TAG_NEVER)
+        dimg, himg = dev.poison_img(gi.TAG_NEVER), host.poison_img(gi.TAG_NEVER)
+        dc, do = dev.alloc(sh, 37)
+        fill_blocks(dev, dimg, sh, do, [(0, j) for j in range(37)])
+        hc, ho = host.alloc(sh, 37)
+        x = ctx.kv_swap_out(sh.as_tuple(), dc, hc)
+        ctx.layer_ready(x, -1, aeg.READY_BLOCK)
+        himg = OK.swap_out(dimg, dev.geom, himg, host.geom, sh, do, ho)
+        assert first_diff(host.read(), himg) is None
+        nc, no = dev.alloc(sh, 37)
+        y = ctx.kv_swap_in(sh.as_tuple(), hc, nc)
+        ctx.layer_ready(y, -1, aeg.READY_BLOCK)
+        dimg = OK.swap_in(himg, host.geom, dimg, dev.geom, sh, ho, no)
+        assert first_diff(dev.read(), dimg) is None
+    finally:
+        ctx.shutdown()
+
+
+def test_invalid_shapes_and_sizes():
+    require_gpu()
+    ctx, dev, host = make(slot=MIB)
+    try:
+        with pytest.raises(aeg.AegError) as e:
+            ctx.kv_alloc(0, (2, 1, 3, 2, 1), 1)          # chunk 12 B: not a multiple of 16
+        assert e.value.code == aeg.ERR_INVALID
+        big = (1, 9, 128, 2, 256)                         # chunk = 256*2*9*128*2 B = 1.125 MiB
+        with pytest.raises(aeg.AegError) as e:
+            ctx.kv_alloc(0, big, 1)                       # block larger than a 1 MiB slab
+        assert e.value.code == aeg.ERR_INVALID
+    finally:
+        ctx.shutdown()
+    ctx, dev, host = make(slot=MIB, slab=4 * MIB)
+    try:
+        big = (1, 9, 128, 2, 256)                         # 1.125 MiB chunk > 1 MiB staging slot
+        d = ctx.kv_alloc(0, big, 1)
+        h = ctx.kv_alloc(1, big, 1)
+        with pytest.raises(aeg.AegError) as e:
+            ctx.kv_swap_out(big, d, h)
+        assert e.value.code == aeg.ERR_INVALID
+        # the migrate kernel has no staging: it accepts the big chunk
+        d2 = ctx.kv_alloc(0, big, 1)
+        x = ctx.kv_migrate(big, d, -1, d2)
+        ctx.layer_ready(x, -1, aeg.READY_BLOCK)
+    finally:
+        ctx.shutdown()
+
+
+def test_oom_changes_nothing_and_release_semantics():
+    require_gpu()
+    ctx, dev, host = make()
+    try:
+        sh = (2, 2, 64, 2, 16)
+        a = ctx.kv_alloc(0, sh, 10)
+        before = ctx.stats(0)
+        with pytest.raises(aeg.AegError) as e:
+            ctx.kv_alloc(0, sh, 1000)
+        assert e.value.code == aeg.ERR_OOM
+        after = ctx.stats(0)
+        assert (after.owned_blocks, after.free_slabs) == (before.owned_blocks, before.free_slabs)
+        h = ctx.kv_alloc(1, sh, 10)
+        x = ctx.kv_swap_out(sh, a, h)
+        ctx.layer_ready(x, -1, aeg.READY_BLOCK)
+        ctx.xfer_release(x)
+        with pytest.raises(aeg.AegError) as e:
+            ctx.layer_ready(x, 0, aeg.READY_QUERY)       # released
+        assert e.value.code == aeg.ERR_STATE
+        with pytest.raises(aeg.AegError) as e:
+            ctx.layer_ready(987654, 0, aeg.READY_QUERY)  # unknown
+        assert e.value.code == aeg.ERR_STATE
+        y = ctx.kv_swap_in(sh, h, a)
+        with pytest.raises(aeg.AegError) as e:
+            ctx.layer_ready(y, 2, aeg.READY_QUERY)       # layer out of range
+        assert e.value.code == aeg.ERR_INVALID
+        ctx.layer_ready(y, -1, aeg.READY_BLOCK)
+    finally:
+        ctx.shutdown()
+
+
+def test_swap_sources_must_be_owned_and_distinct():
+    require_gpu()
+    ctx, dev, host = make()
+    try:
+        sh = (2, 2, 64, 2, 16)
+        a = ctx.kv_alloc(0, sh, 4)
+        h = ctx.kv_alloc(1, sh, 4)
+        with pytest.raises(aeg.AegError) as e:
+            ctx.kv_swap_out(sh, np.array([a[0], a[0], a[1], a[2]], np.uint64), h)
+        assert e.value.code == aeg.ERR_STATE
+        with pytest.raises(aeg.AegError) as e:
+            ctx.kv_swap_out(sh, h, a)                    # pools swapped
+        assert e.value.code == aeg.ERR_INVALID
+        ctx.kv_free(0, a)
+        with pytest.raises(aeg.AegError) as e:
+            ctx.kv_swap_out(sh, a, h)                    # freed sources
+        assert e.value.code in (aeg.ERR_STATE, aeg.ERR_INVALID)
+    finally:
+        ctx.shutdown()

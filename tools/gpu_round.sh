@@ -5,7 +5,7 @@ mkdir -p gpurun_out
 what="${*:-tests bench ncu}"
 nvidia-smi --query-gpu=clocks.sm,clocks.max.sm --format=csv > gpurun_out/clocks_start.csv 2>&1
 if [[ $what == *tests* ]]; then
-  timeout 900 python -m pytest tests -m gpu -q -p no:cacheprovider --timeout 300 -rA > gpurun_out/gpu_tests.log 2>&1
+  timeout 900 python -m pytest tests -m gpu -q -p no:cacheprovider --timeout 300 --timeout-method thread -rA > gpurun_out/gpu_tests.log 2>&1
   echo "pytest rc=$?" >> gpurun_out/gpu_tests.log
   timeout 180 python -c "import __graft_entry__ as g; g.smoke()" > gpurun_out/smoke.log 2>&1; echo "smoke rc=$?" >> gpurun_out/smoke.log
 fi
