@@ -489,6 +489,7 @@ def switch_leg(aeg, torch, n_switch, kernel, descs, mode="staged", caches=None):
         pre = (names[1], xp, int(o[0]))
     cons = torch.cuda.Stream()
     res = []
+    diag_ms = None
     order = [names[(i + 1) % len(names)] for i in range(n_switch + 3)]
     for i, nxt in enumerate(order):
         if pre is not None:   # the decode turn of `cur` hides the prefetch
@@ -512,6 +513,16 @@ def switch_leg(aeg, torch, n_switch, kernel, descs, mode="staged", caches=None):
         db = ctx.kv_alloc(aeg.POOL_DEVICE, nsh, kv[nxt][1])
         xi = ctx.kv_swap_in(nsh, kv[nxt][0], db, flags=aeg.FREE_SRC)                  # B's KV in
         kv[nxt] = (db, kv[nxt][1])
+        diag = {}
+        if i == 3:   # one switch: when does each piece land (device timeline, separate streams)?
+            for name, (xx, l) in {"weights_l0": (xw, wl(0)), "weights_l1": (xw, wl(1)), "kv_l0": (xi, 0),
+                                  "kv_last": (xi, nsh[0] - 1), "kv_out_all": (xo, -1), "weights_all": (xw, -1)
+                                  }.items():
+                ds = torch.cuda.Stream()
+                ctx.layer_ready(xx, l, aeg.READY_WAIT_STREAM, ds.cuda_stream)
+                de = torch.cuda.Event(enable_timing=True)
+                de.record(ds)
+                diag[name] = de
         ev = []
         for l in range(nsh[0]):
             if l == 0:
@@ -529,6 +540,10 @@ def switch_leg(aeg, torch, n_switch, kernel, descs, mode="staged", caches=None):
             ctx.layer_ready(xx, -1, aeg.READY_BLOCK)
             ctx.xfer_release(xx)
         kvb = kv[nxt][1] * nsh[0] * 2 * nsh[1] * nsh[2] * nsh[3] * nsh[4]
+        if diag:
+            torch.cuda.synchronize()
+            diag_ms = {k: round(e0.elapsed_time(v), 2) for k, v in diag.items()}
+            diag_ms["to"] = nxt
         if i >= 3:
             res.append(dict(to=nxt, first_ms=e0.elapsed_time(ev[0]), last_ms=e0.elapsed_time(e_end),
                             bytes_h2d=(0 if mode == "prefetch" else wsize[nxt]) + kvb))
@@ -572,7 +587,8 @@ def switch_leg(aeg, torch, n_switch, kernel, descs, mode="staged", caches=None):
            "direct": "weights DMA'd straight from the page-locked Model Cache (registered once)",
            "prefetch": "weights prefetched during the previous turn, relocated on-device at the switch (3.b)"}[mode]
     return {"workload": f"configs[3] 3-model switch (Qwen-1.8B, Llama-7B, Yi-9B shapes), 1 GiB KV each; {how}",
-            "per_model": per, "weights_bit_exact_sample": bad == 0, "register_s": reg_s}
+            "per_model": per, "weights_bit_exact_sample": bad == 0, "register_s": reg_s,
+            "landing_ms_one_switch": diag_ms}
 
 
 def migrate_leg(aeg, torch, kernel, n_req=4):

@@ -158,12 +158,17 @@ def _decode_host_route_body(conn):
     """Decode instance of Fig. 10: imports the prefill instance's shared CPU cache and its swap-out
     events, swaps R1 in from there (C->D) without any host synchronisation on the prefill side's
     progress, and exports its swap-in so the prefill side can release the CPU blocks."""
+    import sys
     ctx, dev = make(aeg.LAYER_MAJOR, slab=MIB, nslabs=4)
     dev.poison(gi.TAG_NEVER)
+    # connect once at start-up (mapping a peer's pool / registering its shared host region may wait
+    # for the GPU to drain, so it must not sit on the critical path of a hand-off)
+    ctx.import_peer(0, conn.recv())
     conn.send("ready")
-    blob_pool, hb, xblob = conn.recv()
-    ctx.import_peer(0, blob_pool)
+    hb, xblob = conn.recv()
+    print("decode: got hand-off", file=sys.stderr, flush=True)
     xo = ctx.xfer_import(0, xblob)
+    print("decode: imported events", file=sys.stderr, flush=True)
     dc, do = dev.alloc(SH, len(hb))
     xi = ctx.kv_swap_in_from(SH.as_tuple(), 0, np.array(hb, dtype=np.uint64), dc, after=xo)   # ③④⑤
     conn.send((ctx.xfer_export(xi), do))
@@ -208,14 +213,15 @@ def test_two_process_host_route_p_c_d():
         sc, so = A.alloc(SH, 20)
         fill_blocks(A, aimg, SH, so, [(1, j) for j in range(20)])
         hc, ho = H.alloc(SH, 20)
-        assert recv() == "ready"                      # the decode instance is up
+        parent.send(a.export_ipc())                   # instances connect at start-up
+        assert recv() == "ready"                      # the decode instance is up and connected
         s = torch.cuda.Stream()
         from aeg_inputs import dev as Dv
         gate = Dv.Gate()
         gate.close_on(s.cuda_stream)                  # the prefill is still running until gate.open()
         a.stream_fence(s.cuda_stream)
         xo = a.kv_swap_out(SH.as_tuple(), sc, hc, flags=aeg.FREE_SRC)                            # ①②
-        parent.send((a.export_ipc(), [int(b) for b in hc], a.xfer_export(xo)))
+        parent.send(([int(b) for b in hc], a.xfer_export(xo)))
         xblob, do = recv()
         xd = a.xfer_import(1, xblob)
         out_done = a.layer_ready(xo, -1, aeg.READY_QUERY)
