@@ -206,7 +206,28 @@ cudaError_t launch_t(const CopyArgs& a, int impl, int max_ctas, cudaStream_t s) 
   return cudaGetLastError();
 }
 
+template <bool SP, bool DP>
+cudaError_t preload_t() {
+  cudaFuncAttributes fa;
+  cudaError_t e = cudaFuncGetAttributes(&fa, copy_lsu<SP, DP>);
+  if (e == cudaSuccess) e = cudaFuncGetAttributes(&fa, copy_bulk<SP, DP>);
+  if (e == cudaSuccess)
+    e = cudaFuncSetAttribute(copy_bulk<SP, DP>, cudaFuncAttributeMaxDynamicSharedMemorySize, kBulkSmem);
+  return e;
+}
+
 }  // namespace
+
+// Load every copy kernel into the current device's context now.  With CUDA's lazy module loading a
+// kernel's first launch loads its module and waits for the device; on the hot path that is both a
+// latency spike and a deadlock hazard when another kernel spin-waits (found by the gate tests).
+cudaError_t preload_kernels() {
+  cudaError_t e = preload_t<true, false>();
+  if (e == cudaSuccess) e = preload_t<false, true>();
+  if (e == cudaSuccess) e = preload_t<true, true>();
+  if (e == cudaSuccess) e = preload_t<false, false>();
+  return e;
+}
 
 cudaError_t launch_copy(const CopyArgs& a, int impl, int max_ctas, cudaStream_t s) {
   const bool sp = a.src_off != nullptr, dp = a.dst_off != nullptr;

@@ -31,6 +31,9 @@ enum CopyImpl { IMPL_LSU = 1, IMPL_BULK = 2 };
 // (cp.async.bulk global->smem->global, mbarrier pipeline, one issuing thread per CTA).
 cudaError_t launch_copy(const CopyArgs& a, int impl, int max_ctas, cudaStream_t s);
 
+// Load all copy kernels (and set the BULK shared-memory attribute) for the current device.
+cudaError_t preload_kernels();
+
 // memmove inside one buffer (N1): overlap-safe ascending / descending chunking.
 cudaError_t launch_memmove(char* base, uint64_t src_off, uint64_t dst_off, uint64_t bytes, int impl,
                            cudaStream_t s, int* launches);

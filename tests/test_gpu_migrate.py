@@ -170,8 +170,12 @@ def _decode_host_route_body(conn):
     xo = ctx.xfer_import(0, xblob)
     print("decode: imported events", file=sys.stderr, flush=True)
     dc, do = dev.alloc(SH, len(hb))
+    print("decode: allocated", file=sys.stderr, flush=True)
     xi = ctx.kv_swap_in_from(SH.as_tuple(), 0, np.array(hb, dtype=np.uint64), dc, after=xo)   # ③④⑤
-    conn.send((ctx.xfer_export(xi), do))
+    print("decode: swap-in enqueued", file=sys.stderr, flush=True)
+    blob = ctx.xfer_export(xi)
+    print("decode: exported", file=sys.stderr, flush=True)
+    conn.send((blob, do))
     for l in range(SH.L):
         ctx.layer_ready(xi, l, aeg.READY_BLOCK)                                                  # ⑥
     conn.send(dev.read().tobytes())
