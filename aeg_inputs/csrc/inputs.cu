@@ -213,6 +213,20 @@ int aegin_copy(void* dst, const void* src, uint64_t n) { return int(cudaMemcpy(d
 
 int aegin_sync(void) { return int(cudaDeviceSynchronize()); }
 
+// Load every kernel of this library now (no lazy module load later, which would wait for a
+// running gate kernel and deadlock a race test).
+int aegin_preload(void) {
+  cudaFuncAttributes a;
+  cudaError_t e = cudaFuncGetAttributes(&a, fill_chunks);
+  if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, verify_chunks);
+  if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, fill_region);
+  if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, verify_region);
+  if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, consume_chunks);
+  if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, gate);
+  if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, spin);
+  return int(e);
+}
+
 int aegin_gate(const void* pinned_flag, void* stream) {
   gate<<<1, 1, 0, static_cast<cudaStream_t>(stream)>>>(static_cast<const volatile int*>(pinned_flag));
   return int(cudaGetLastError());

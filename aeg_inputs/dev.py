@@ -28,6 +28,7 @@ def lib():
             "aegin_consume": [P, P, U64, U64, P, P],
             "aegin_spin": [C.c_longlong, P],
             "aegin_gate": [P, P],
+            "aegin_preload": [],
             "aegin_copy": [P, P, U64],
             "aegin_sync": [],
             "aegin_host_fill": [P, U64, U64, U64, C.c_int],
@@ -36,6 +37,9 @@ def lib():
             getattr(L, k).argtypes = a
             getattr(L, k).restype = C.c_int
         _L = L
+        rc = L.aegin_preload()
+        if rc not in (0, 35, 100):      # 35/100: no driver / no device (CPU-only box)
+            _ck(rc)
     return _L
 
 

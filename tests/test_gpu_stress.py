@@ -1,0 +1,128 @@
+"""Race stress (SURVEY.md §4 race tests; rules ❶❷❸): seeded random sequences of
+swap-out / swap-in / local migrate / free (with FREE_SRC move lists) over small pools, while gate
+kernels hold some transfers back and open at random later points, so transfers overlap in every
+order the rules allow.  Checks: (1) the library's own primitive log passes the oracle's
+happens-before checker (oracle/rules.py), including consumer reads after per-layer waits (❶);
+(2) the final device and host images equal the oracle's sequential replay (oracle/kv.py) of the same
+operations in host order, at the placements the library chose."""
+import random
+
+import numpy as np
+import pytest
+
+import aeg_inputs as gi
+import paper_conf_sosp_xiang0qyzyzl0025_b200 as aeg
+from aeg_inputs import dev as D
+from oracle import kv as OK
+from oracle.rules import check
+from oracle.shape import KVShape
+
+from .gpu_harness import SEED, Side, first_diff, require_gpu
+from .test_gpu_swap import parse_trace
+
+pytestmark = pytest.mark.gpu
+KIB = 1024
+SH = KVShape(2, 4, 64, 2, 16)            # 16 KiB chunks, 32 KiB blocks
+
+
+def dec(bs):
+    return [aeg.decode_block(b)[1:] for b in bs]
+
+
+@pytest.mark.parametrize("seed", range(6))
+def test_random_overlapping_transfers(seed):
+    require_gpu()
+    import torch
+    r = random.Random(seed)
+    cfg = aeg.default_config(device_kv_bytes=24 * 256 * KIB, host_kv_bytes=24 * 256 * KIB, dev_slab_bytes=256 * KIB,
+                             host_slab_bytes=256 * KIB, dev_slab_layout=seed % 2, host_slab_layout=(seed // 2) % 2,
+                             staging_slot_bytes=1 << 20, staging_slots=2, stage_ring_bytes=4 << 20,
+                             stage_chunk_bytes=1 << 20, device_weight_bytes=2 << 20, table_arena_bytes=2 << 20,
+                             host_threads=1, kernel=aeg.KERNEL_BULK if seed % 3 else aeg.KERNEL_LSU)
+    ctx = aeg.Context(0, cfg)
+    try:
+        dev = Side(ctx, 0, cfg.device_kv_bytes, cfg.dev_slab_bytes, cfg.dev_slab_layout)
+        host = Side(ctx, 1, cfg.host_kv_bytes, cfg.host_slab_bytes, cfg.host_slab_layout)
+        dev.poison(gi.TAG_NEVER)
+        host.poison(gi.TAG_NEVER)
+        dimg, himg = dev.poison_img(gi.TAG_NEVER), host.poison_img(gi.TAG_NEVER)
+        log = []
+        ctx.trace_enable(True)
+
+        def flush():
+            log.extend(parse_trace(ctx.trace_read()))
+
+        objs = []        # [where, handles]
+        gates = []       # open gates
+        cons = torch.cuda.Stream()
+        for step in range(45):
+            op = r.choice(["new", "new", "out", "out", "in", "in", "mig", "free", "gate", "open", "use"])
+            if op == "new" or not objs:
+                n = r.randint(1, 12)
+                try:
+                    c = ctx.kv_alloc(0, SH.as_tuple(), n)
+                except aeg.AegError:
+                    continue
+                offs, keys = [], []
+                for j, h in enumerate(dec(c)):
+                    for l in range(SH.L):
+                        o = OK.addr(dev.geom, SH, h, l)
+                        offs.append(o)
+                        keys.append(gi.kv_key(2, step, j, l))
+                        dimg[o:o + SH.chunk_bytes()] = gi.region_bytes(SEED, keys[-1], SH.chunk_bytes())
+                D.fill_chunks(dev.base, offs, keys, SH.chunk_bytes(), SEED)
+                # fresh blocks are touched by no incomplete transfer (❸); log the fill as a write
+                flush()
+                log.append(("op", "fill", "fill", [], [f"D:{s}:{j}:{l}" for s, j in dec(c) for l in range(SH.L)]))
+                objs.append(["dev", c])
+                continue
+            o = r.choice(objs)
+            try:
+                if op == "out" and o[0] == "dev":
+                    hc = ctx.kv_alloc(1, SH.as_tuple(), len(o[1]))
+                    ctx.kv_swap_out(SH.as_tuple(), o[1], hc, flags=aeg.FREE_SRC)
+                    himg = OK.swap_out(dimg, dev.geom, himg, host.geom, SH, dec(o[1]), dec(hc))
+                    o[:] = ["host", hc]
+                elif op == "in" and o[0] == "host":
+                    dc = ctx.kv_alloc(0, SH.as_tuple(), len(o[1]))
+                    x = ctx.kv_swap_in(SH.as_tuple(), o[1], dc, flags=aeg.FREE_SRC)
+                    dimg = OK.swap_in(himg, host.geom, dimg, dev.geom, SH, dec(o[1]), dec(dc))
+                    o[:] = ["dev", dc, x]
+                elif op == "mig" and o[0] == "dev":
+                    dc = ctx.kv_alloc(0, SH.as_tuple(), len(o[1]))
+                    x = ctx.kv_migrate(SH.as_tuple(), o[1], -1, dc, flags=aeg.FREE_SRC)
+                    dimg = OK.migrate(dimg, dev.geom, dimg, dev.geom, SH, dec(o[1]), dec(dc))
+                    o[:] = ["dev", dc, x]
+                elif op == "free":
+                    ctx.kv_free(0 if o[0] == "dev" else 1, o[1])
+                    objs.remove(o)
+                elif op == "gate":
+                    s = torch.cuda.Stream()
+                    g = D.Gate()
+                    g.close_on(s.cuda_stream)
+                    ctx.stream_fence(s.cuda_stream)     # later transfers wait until it opens
+                    gates.append(g)
+                elif op == "open" and gates:
+                    gates.pop(r.randrange(len(gates))).open()
+                elif op == "use" and o[0] == "dev" and len(o) > 2:
+                    # rule ❶: a decode consumer waits per layer on the transfer that produced o, then reads
+                    for l in range(SH.L):
+                        ctx.layer_ready(o[2], l, aeg.READY_WAIT_STREAM, cons.cuda_stream)
+                    flush()
+                    log.append(("use", "u0x%x" % cons.cuda_stream,
+                                [f"D:{s}:{j}:{l}" for s, j in dec(o[1]) for l in range(SH.L)]))
+            except aeg.AegError as e:
+                assert e.code == aeg.ERR_OOM, e       # pools are small: OOM is the only legal refusal
+            flush()
+        for g in gates:
+            g.open()
+        ctx.reclaim(blocking=True)
+        torch.cuda.synchronize()
+        flush()
+        assert check(log)
+        assert first_diff(dev.read(), dimg) is None
+        assert first_diff(host.read(), himg) is None
+    finally:
+        for g in locals().get("gates", []):
+            g.open()
+        ctx.shutdown()
