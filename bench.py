@@ -500,6 +500,12 @@ def switch_leg(aeg, torch, n_switch, kernel, descs, mode="staged", caches=None):
         hb = ctx.kv_alloc(aeg.POOL_HOST, shapes[cur], kv[cur][1])
         xo = ctx.kv_swap_out(shapes[cur], kv[cur][0], hb, flags=aeg.FREE_SRC)        # A's KV out (D2H)
         kv[cur] = (hb, kv[cur][1])
+        # B's KV goes first: the copy engine serves one busy H2D stream until it drains
+        # (profiles/r01/ce_probe.txt), so KV queued behind a model's weights would land last
+        nsh = shapes[nxt]
+        db = ctx.kv_alloc(aeg.POOL_DEVICE, nsh, kv[nxt][1])
+        xi = ctx.kv_swap_in(nsh, kv[nxt][0], db, flags=aeg.FREE_SRC)                  # B's KV in
+        kv[nxt] = (db, kv[nxt][1])
         if mode in ("staged", "direct"):
             ctx.weights_reset(0)
             _, xw = ctx.weights_stage(descs[nxt])                                      # B's weights in
@@ -509,10 +515,6 @@ def switch_leg(aeg, torch, n_switch, kernel, descs, mode="staged", caches=None):
             xw = ctx.weights_relocate(pre[2], 0, wsize[nxt])                           # 3.b: on-device copy
             ctx.xfer_release(pre[1])
             wl = lambda l: 0  # noqa: E731
-        nsh = shapes[nxt]
-        db = ctx.kv_alloc(aeg.POOL_DEVICE, nsh, kv[nxt][1])
-        xi = ctx.kv_swap_in(nsh, kv[nxt][0], db, flags=aeg.FREE_SRC)                  # B's KV in
-        kv[nxt] = (db, kv[nxt][1])
         diag = {}
         if i == 3:   # one switch: when does each piece land (device timeline, separate streams)?
             for name, (xx, l) in {"weights_l0": (xw, wl(0)), "weights_l1": (xw, wl(1)), "kv_l0": (xi, 0),

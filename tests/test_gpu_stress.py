@@ -73,10 +73,14 @@ def test_random_overlapping_transfers(seed):
                 D.fill_chunks(dev.base, offs, keys, SH.chunk_bytes(), SEED)
                 # fresh blocks are touched by no incomplete transfer (❸); log the fill as a write
                 flush()
+                # the fill is synchronous: the host saw it complete before issuing anything later
                 log.append(("op", "fill", "fill", [], [f"D:{s}:{j}:{l}" for s, j in dec(c) for l in range(SH.L)]))
+                log.append(("record", "fill", f"fill{step}"))
+                log.append(("sync", f"fill{step}"))
                 objs.append(["dev", c])
                 continue
-            o = r.choice(objs)
+            oi = r.randrange(len(objs))
+            o = objs[oi]
             try:
                 if op == "out" and o[0] == "dev":
                     hc = ctx.kv_alloc(1, SH.as_tuple(), len(o[1]))
@@ -95,7 +99,7 @@ def test_random_overlapping_transfers(seed):
                     o[:] = ["dev", dc, x]
                 elif op == "free":
                     ctx.kv_free(0 if o[0] == "dev" else 1, o[1])
-                    objs.remove(o)
+                    del objs[oi]
                 elif op == "gate":
                     s = torch.cuda.Stream()
                     g = D.Gate()
