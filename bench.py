@@ -517,8 +517,9 @@ def switch_leg(aeg, torch, n_switch, kernel, descs, mode="staged", caches=None):
             wl = lambda l: 0  # noqa: E731
         diag = {}
         if i == 3:   # one switch: when does each piece land (device timeline, separate streams)?
-            for name, (xx, l) in {"weights_l0": (xw, wl(0)), "weights_l1": (xw, wl(1)), "kv_l0": (xi, 0),
-                                  "kv_last": (xi, nsh[0] - 1), "kv_out_all": (xo, -1), "weights_all": (xw, -1)
+            # KV probes first: a weights-layer wait blocks the host until the pipeline records it
+            for name, (xx, l) in {"kv_l0": (xi, 0), "kv_last": (xi, nsh[0] - 1), "kv_out_all": (xo, -1),
+                                  "weights_l0": (xw, wl(0)), "weights_l1": (xw, wl(1)), "weights_all": (xw, -1)
                                   }.items():
                 ds = torch.cuda.Stream()
                 ctx.layer_ready(xx, l, aeg.READY_WAIT_STREAM, ds.cuda_stream)

@@ -264,6 +264,9 @@ int aeg_xfer_release(aeg_ctx ctx, aeg_xfer x);
  * dev_offsets_out[n] receives byte offsets inside the weights region.  Returns after the host
  * pipeline is started; the layer events are recorded as chunks are issued (WAIT_STREAM and
  * BLOCK readiness first wait on the host until the event is recorded).
+ * Composition note (measured): one copy engine serves a busy H2D stream until it
+ * drains, so in a model switch enqueue the incoming KV swap-in BEFORE the weights, or the KV lands
+ * after the whole model.
  * INVALID for non-divisible splits, OOM if the region is exhausted. */
 int aeg_weights_stage(aeg_ctx ctx, const aeg_weight_desc* descs, int32_t n, int32_t tp_rank,
                       int32_t tp_size, uint64_t* dev_offsets_out, aeg_xfer* out);

@@ -348,13 +348,16 @@ class Context:
         _chk(lib().aeg_trace_enable(self.h, int(on)))
 
     def trace_read(self) -> str:
-        n = C.c_uint64(0)
-        rc = lib().aeg_trace_read(self.h, None, C.byref(n))
-        buf = C.create_string_buffer(n.value + 1)
-        n2 = C.c_uint64(n.value + 1)
-        _chk(lib().aeg_trace_read(self.h, buf, C.byref(n2)))
-        del rc
-        return buf.value.decode()
+        """Copy out and clear the primitive trace (the daemon may append between calls: retry)."""
+        for _ in range(100):
+            n = C.c_uint64(0)
+            lib().aeg_trace_read(self.h, None, C.byref(n))      # INVALID by design: returns the size
+            cap = 2 * n.value + 65536
+            buf = C.create_string_buffer(cap)
+            n2 = C.c_uint64(cap)
+            if lib().aeg_trace_read(self.h, buf, C.byref(n2)) == OK:
+                return buf.raw[: n2.value].decode()
+        raise AegError(ERR_STATE, "trace kept growing")
 
     def debug_xfer_begin(self, pool: int, blocks) -> int:
         b = _blocks(blocks)
