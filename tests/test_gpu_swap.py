@@ -183,3 +183,36 @@ def test_kernel_timing_counters():
         assert n >= 1 and b == 2 * len(do) * SH.block_bytes() and ms > 0
     finally:
         ctx.shutdown()
+
+
+def test_layer_readiness_is_monotone_and_live():
+    """O9: every layer of a swap eventually becomes ready (liveness) and, once
+    QUERY reports it ready, it stays ready (monotonicity); layer l never reports ready while its bytes
+    differ from the oracle (safety: checked right after the first ready observation)."""
+    require_gpu()
+    ctx, dev, host = make(aeg.LAYER_MAJOR, aeg.LAYER_MAJOR, aeg.KERNEL_BULK, 1 << 20)
+    try:
+        dev.poison(gi.TAG_NEVER)
+        host.poison(gi.TAG_NEVER)
+        dimg, himg = dev.poison_img(gi.TAG_NEVER), host.poison_img(gi.TAG_NEVER)
+        dc, do = requests(dev, dimg, SH)
+        hc, ho = host.alloc(SH, len(do))
+        x = ctx.kv_swap_out(SH.as_tuple(), dc, hc)
+        himg = OK.swap_out(dimg, dev.geom, himg, host.geom, SH, do, ho)
+        seen = [False] * SH.L
+        for _ in range(1_000_000):
+            for l in range(SH.L):
+                r = ctx.layer_ready(x, l, aeg.READY_QUERY)
+                assert r or not seen[l]
+                if r and not seen[l]:
+                    seen[l] = True
+                    got = host.read()
+                    for h in ho:
+                        o = OK.addr(host.geom, SH, h, l)
+                        assert np.array_equal(got[o:o + SH.chunk_bytes()], himg[o:o + SH.chunk_bytes()])
+            if all(seen):
+                break
+        assert all(seen)
+        assert ctx.layer_ready(x, -1, aeg.READY_QUERY) or ctx.layer_ready(x, -1, aeg.READY_BLOCK)
+    finally:
+        ctx.shutdown()

@@ -32,8 +32,8 @@ def model_cache(descs, m=1):
     return buf, tens
 
 
-def synth_model(h=512, L=4, ff=1536, V=4096):
-    gi.MODELS["_test"] = (h, L, ff, V, h // 4, "llama")
+def synth_model(h=512, L=4, ff=1536, V=4096, arch="llama"):
+    gi.MODELS["_test"] = (h, L, ff, V, h // 4, arch)
     d = gi.model_tensors("_test")
     del gi.MODELS["_test"]
     return d
@@ -54,9 +54,10 @@ def descs_for(buf_tens, descs):
 
 @pytest.mark.parametrize("tp", [1, 2, 4])
 @pytest.mark.parametrize("direct", [False, True])
-def test_stage_matches_oracle(tp, direct):
+@pytest.mark.parametrize("arch", ["llama", "qwen1"])      # qwen1: fused QKV, COL split per group of 3
+def test_stage_matches_oracle(tp, direct, arch):
     require_gpu()
-    descs = synth_model()
+    descs = synth_model(arch=arch)
     buf, tens = model_cache(descs)
     ctx = make()
     try:
