@@ -338,9 +338,15 @@ uint64_t Ctx::migrate(const Shape& sh, const aeg_block* src, int32_t peer, const
     for (int32_t i = 0; i < n; ++i) t[n + i] = dg->off0(dst[i], sh);
     CUDA_TRY(cudaMemcpyAsync(dtab, htab, uint64_t(n) * 16, cudaMemcpyHostToDevice, s_migrate));
   }
+  // Layers per launch: every launch pays a fixed ~8-36 us, so pack layers up to a
+  // target payload.  Same-device destinations copy at HBM speed (a 133 MiB layer is ~45 us): pack to
+  // 512 MiB.  Over NVLink a 128 MiB launch already takes ~170 us, and per-layer readiness lets the
+  // decode instance start early, so remote destinations keep (at least) one launch per 128 MiB.
+  const bool remote = P && (!P->same_process || P->device != device);
+  const uint64_t pack = remote ? (128ull << 20) : (512ull << 20);
   const uint64_t layer = uint64_t(n) * sh.chunk();
   int32_t lps = 1;
-  if (n > 0 && layer < kPackLayerBytes) lps = int32_t(std::min<uint64_t>(sh.L, std::max<uint64_t>(1, kPackLayerBytes / layer)));
+  if (n > 0 && layer < pack) lps = int32_t(std::min<uint64_t>(sh.L, std::max<uint64_t>(1, pack / layer)));
   const int impl = (P && !P->same_process && cfg.kernel == AEG_KERNEL_AUTO) || (P && P->device != device && cfg.kernel == AEG_KERNEL_AUTO)
                        ? IMPL_LSU : impl_of(cfg);
   for (int32_t la = 0; la < sh.L; la += lps) {
