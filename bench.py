@@ -296,10 +296,10 @@ class SwapBench:
         self.lab[(offs // np.uint64(self.Cl)).astype(np.int64)] = keys
 
     def consumer_tables(self, torch, blocks):
-        """[L][n] byte offsets of each layer of `blocks` from the pool base (via aeg_block_ptr)."""
-        p0 = np.array([self.ctx.block_ptr(0, self.sht, int(b), 0) for b in blocks], dtype=np.uint64)
-        stride = self.ctx.block_ptr(0, self.sht, int(blocks[0]), 1) - int(p0[0])
-        t = (p0 - np.uint64(self.dbase))[None, :] + np.arange(self.sh.L, dtype=np.uint64)[:, None] * np.uint64(stride)
+        """[L][n] byte offsets of each layer of `blocks` from the pool base (aeg_block_offsets: the
+        block table a PagedAttention-style consumer would build)."""
+        off0, stride = self.ctx.block_offsets(0, self.sht, blocks)
+        t = off0[None, :] + np.arange(self.sh.L, dtype=np.uint64)[:, None] * np.uint64(stride)
         return torch.from_numpy(t.astype(np.int64)).cuda()
 
     def step(self, torch, cons, with_consumer=True, record=True):
@@ -911,6 +911,12 @@ def run_ours(args):
             "consumer_launches": args.steps * sb.sh.L,
         }
         res.update(out)
+        od = out.get("one_direction")
+        if od:   # each direction alone against PCIe Gen5 x16 nominal 64 GB/s (target >= 0.80)
+            res["pcie"]["swap_out_alone_GBps"] = od["swap_out"]["GBps"]
+            res["pcie"]["swap_in_alone_GBps"] = od["swap_in"]["GBps"]
+            res["pcie"]["swap_out_alone_frac"] = round(od["swap_out"]["GBps"] / PCIE_NOMINAL, 3)
+            res["pcie"]["swap_in_alone_frac"] = round(od["swap_in"]["GBps"] / PCIE_NOMINAL, 3)
         print(json.dumps(res), flush=True)
     dist.close()
     return 0

@@ -189,6 +189,13 @@ int aeg_block_info(aeg_ctx ctx, aeg_block b, int32_t* pool, uint32_t* slab, uint
 int aeg_block_ptr(aeg_ctx ctx, int32_t pool, const aeg_kv_shape* shape, aeg_block b,
                   int32_t layer, void** p);
 
+/* Block table for a consumer (e.g. a PagedAttention kernel): off0[i] = byte offset of layer 0 of
+ * blocks[i] from the pool base, and *layer_stride = bytes between consecutive layers of a block (the
+ * same for every block of `shape` in this pool), so layer l of block i is at base + off0[i] +
+ * l * layer_stride.  All blocks must be owned and of `shape`.  O(n), one call. */
+int aeg_block_offsets(aeg_ctx ctx, int32_t pool, const aeg_kv_shape* shape, const aeg_block* blocks,
+                      int32_t n, uint64_t* off0, uint64_t* layer_stride);
+
 /* Base pointer and size of a pool's region (device pointer for DEVICE, host pointer for HOST). */
 int aeg_pool_region(aeg_ctx ctx, int32_t pool, void** base, uint64_t* bytes);
 

@@ -97,6 +97,7 @@ _SIGS = {
     "aeg_block_info": [P, U64, PI32, PU32, PU32],
     "aeg_block_ptr": [P, I32, C.POINTER(KVShape), U64, I32, C.POINTER(P)],
     "aeg_pool_region": [P, I32, C.POINTER(P), PU64],
+    "aeg_block_offsets": [P, I32, C.POINTER(KVShape), PU64, I32, PU64, PU64],
     "aeg_kv_swap_out": [P, C.POINTER(KVShape), PU64, PU64, I32, U32, PU64],
     "aeg_kv_swap_in": [P, C.POINTER(KVShape), PU64, PU64, I32, U32, PU64],
     "aeg_kv_migrate": [P, C.POINTER(KVShape), PU64, I32, PU64, I32, U32, PU64],
@@ -222,6 +223,15 @@ class Context:
         sh = KVShape.of(shape)
         _chk(lib().aeg_block_ptr(self.h, pool, C.byref(sh), int(b), int(layer), C.byref(p)))
         return p.value or 0
+
+    def block_offsets(self, pool: int, shape, blocks):
+        """(layer-0 byte offsets from the pool base [n], per-layer stride) for a consumer's block table."""
+        b = _blocks(blocks)
+        off = np.zeros(max(1, b.size), dtype=np.uint64)
+        stride = C.c_uint64()
+        sh = KVShape.of(shape)
+        _chk(lib().aeg_block_offsets(self.h, pool, C.byref(sh), _p64(b), int(b.size), _p64(off), C.byref(stride)))
+        return off[: b.size], stride.value
 
     def pool_region(self, pool: int):
         p, n = P(), C.c_uint64()

@@ -225,6 +225,21 @@ int aeg_block_ptr(aeg_ctx ctx, int32_t pool, const aeg_kv_shape* shape, aeg_bloc
   });
 }
 
+int aeg_block_offsets(aeg_ctx ctx, int32_t pool, const aeg_kv_shape* shape, const aeg_block* blocks, int32_t n,
+                      uint64_t* off0, uint64_t* layer_stride) {
+  return guarded([&] {
+    Ctx& c = C(ctx);
+    AEG_REQUIRE(pool == AEG_POOL_DEVICE || pool == AEG_POOL_HOST, AEG_ERR_INVALID, "bad pool %d", pool);
+    AEG_REQUIRE((n == 0 || off0) && layer_stride, AEG_ERR_INVALID, "NULL output");
+    const aeg::Shape sh = aeg::Shape::from(shape);
+    std::lock_guard<std::mutex> g(c.mu);
+    c.pool[pool].check_owned(blocks, n, &sh, false);
+    for (int32_t i = 0; i < n; ++i) off0[i] = c.pool[pool].off0(blocks[i], sh);
+    *layer_stride = c.pool[pool].lstride(sh);
+    return AEG_OK;
+  });
+}
+
 int aeg_pool_region(aeg_ctx ctx, int32_t pool, void** base, uint64_t* bytes) {
   return guarded([&] {
     Ctx& c = C(ctx);

@@ -174,6 +174,29 @@ def test_error_codes_and_validation():
     c.shutdown()
 
 
+@pytest.mark.parametrize("layout", [aeg.LAYER_MAJOR, aeg.BLOCK_MAJOR])
+def test_block_offsets_match_oracle_addr(layout):
+    """aeg_block_offsets (the consumer's block table) places every layer of every block exactly where
+    the oracle's address function (O3 geometry) does, for both slab layouts."""
+    from oracle import kv as OK
+    slab = 1 << 20
+    c = host_ctx(8, layout)
+    c.shutdown()
+    cfg = aeg.default_config(device_kv_bytes=8 * slab, host_kv_bytes=8 * slab, dev_slab_bytes=slab,
+                             host_slab_bytes=slab, dev_slab_layout=layout, host_slab_layout=layout,
+                             flags=aeg.CFG_HOST_ONLY | aeg.CFG_NO_DAEMON)
+    c = aeg.Context(0, cfg)
+    sh = KVShape(3, 2, 64, 2, 16)
+    blocks = np.concatenate([c.kv_alloc(0, sh.as_tuple(), 37), c.kv_alloc(0, sh.as_tuple(), 5)])
+    off0, stride = c.block_offsets(0, sh.as_tuple(), blocks)
+    g = OK.PoolGeom(8 * slab, slab, layout)
+    for b, o in zip(blocks, off0):
+        h = aeg.decode_block(b)[1:]
+        for l in range(sh.L):
+            assert int(o) + l * stride == OK.addr(g, sh, h, l)
+    c.shutdown()
+
+
 def test_daemon_reclaims_move_list():
     """With the daemon running, a move-list block is reclaimed without an explicit aeg_reclaim."""
     import time
