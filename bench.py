@@ -463,6 +463,8 @@ def switch_leg(aeg, torch, n_switch, kernel, descs, mode="staged", caches=None):
     region = wmax + 64 * MIB if mode == "staged" else 2 * wmax + 128 * MIB
     cfg = aeg.default_config(device_kv_bytes=8 * GIB, host_kv_bytes=8 * GIB, device_weight_bytes=region,
                              kernel=kernel, host_threads=12)
+    if int(os.environ.get("AEG_STAGE_CHUNK_MIB", "0")):
+        cfg.stage_chunk_bytes = int(os.environ["AEG_STAGE_CHUNK_MIB"]) * MIB
     ctx = aeg.Context(0, cfg)
     reg_s = None
     if mode == "direct":   # page-lock the Model Caches once ("no pinning during scaling")
