@@ -82,7 +82,7 @@ enum {
                                    the node-shared "Unified CPU KV Cache" (Fig. 5) */
 };
 /* kernel selection for gather/scatter/migrate (AEG_KERNEL_AUTO picks the measured best) */
-enum { AEG_KERNEL_AUTO = 0, AEG_KERNEL_LSU = 1, AEG_KERNEL_BULK = 2 };
+enum { AEG_KERNEL_AUTO = 0, AEG_KERNEL_LSU = 1, AEG_KERNEL_BULK = 2, AEG_KERNEL_WARP = 3 };
 
 /* ---- structs ---------------------------------------------------------------------------- */
 

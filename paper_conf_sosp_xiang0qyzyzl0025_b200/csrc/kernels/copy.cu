@@ -85,6 +85,49 @@ __global__ void __launch_bounds__(kLsuThreads) copy_lsu(const CopyArgs a) {
   }
 }
 
+// ------------------------------------------------------------------------------------ WARP
+// Small chunks (<= 8 KiB, e.g. TP-sharded GQA caches with one KV head per rank): a warp takes 32
+// consecutive chunks, each lane resolves one chunk's pointers (one coalesced block-table load per
+// 32 chunks), and the warp then copies the chunks one after another with the pointers broadcast by
+// __shfl_sync — the north star's warp-level index broadcast.
+constexpr int kWarpThreads = 256;
+constexpr int kWarpUnroll = 4;
+
+template <bool SP, bool DP>
+__global__ void __launch_bounds__(kWarpThreads) copy_warp(const CopyArgs a) {
+  const uint64_t total = uint64_t(a.nl) * uint64_t(a.n);
+  const int lane = threadIdx.x & 31;
+  const uint64_t warp = (uint64_t(blockIdx.x) * kWarpThreads + threadIdx.x) >> 5;
+  const uint64_t nwarps = (uint64_t(gridDim.x) * kWarpThreads) >> 5;
+  const uint32_t vecs = uint32_t(a.chunk / 16);
+  for (uint64_t g = warp * 32; g < total; g += nwarps * 32) {
+    const uint64_t c = g + lane;
+    const char* s = nullptr;
+    char* d = nullptr;
+    if (c < total) item_ptrs<SP, DP>(a, c, s, d);
+    const unsigned long long sp = reinterpret_cast<unsigned long long>(s);
+    const unsigned long long dp = reinterpret_cast<unsigned long long>(d);
+    const int cnt = total - g < 32 ? int(total - g) : 32;
+    for (int t = 0; t < cnt; ++t) {
+      const char* st = reinterpret_cast<const char*>(__shfl_sync(0xffffffffu, sp, t));
+      char* dt = reinterpret_cast<char*>(__shfl_sync(0xffffffffu, dp, t));
+      for (uint32_t v0 = 0; v0 < vecs; v0 += 32 * kWarpUnroll) {
+        uint4 x[kWarpUnroll];
+#pragma unroll
+        for (int u = 0; u < kWarpUnroll; ++u) {
+          const uint32_t v = v0 + u * 32 + lane;
+          if (v < vecs) x[u] = ld_stream(st + uint64_t(v) * 16);
+        }
+#pragma unroll
+        for (int u = 0; u < kWarpUnroll; ++u) {
+          const uint32_t v = v0 + u * 32 + lane;
+          if (v < vecs) st_stream(dt + uint64_t(v) * 16, x[u]);
+        }
+      }
+    }
+  }
+}
+
 // ------------------------------------------------------------------------------------ BULK
 constexpr int kBulkStages = 6;
 constexpr uint32_t kBulkPiece = 32768;
@@ -183,7 +226,13 @@ template <bool SP, bool DP>
 cudaError_t launch_t(const CopyArgs& a, int impl, int max_ctas, cudaStream_t s) {
   const uint64_t items_lsu = uint64_t(a.nl) * a.n * ((a.chunk + kLsuPiece - 1) / kLsuPiece);
   if (items_lsu == 0) return cudaSuccess;
-  if (impl == IMPL_BULK) {
+  if (impl == IMPL_WARP) {
+    const uint64_t groups = (uint64_t(a.nl) * a.n + 31) / 32;  // one warp per 32 chunks
+    uint64_t grid = max_ctas > 0 ? uint64_t(max_ctas) : uint64_t(kSMs) * 8;
+    const uint64_t need = (groups * 32 + kWarpThreads - 1) / kWarpThreads;
+    if (grid > need) grid = need;
+    copy_warp<SP, DP><<<unsigned(grid), kWarpThreads, 0, s>>>(a);
+  } else if (impl == IMPL_BULK) {
     static std::atomic<uint64_t> attr_set{0};  // per-device bit: opt-in smem attribute applied
     int dev = 0;
     cudaError_t e = cudaGetDevice(&dev);
@@ -210,6 +259,7 @@ template <bool SP, bool DP>
 cudaError_t preload_t() {
   cudaFuncAttributes fa;
   cudaError_t e = cudaFuncGetAttributes(&fa, copy_lsu<SP, DP>);
+  if (e == cudaSuccess) e = cudaFuncGetAttributes(&fa, copy_warp<SP, DP>);
   if (e == cudaSuccess) e = cudaFuncGetAttributes(&fa, copy_bulk<SP, DP>);
   if (e == cudaSuccess)
     e = cudaFuncSetAttribute(copy_bulk<SP, DP>, cudaFuncAttributeMaxDynamicSharedMemorySize, kBulkSmem);

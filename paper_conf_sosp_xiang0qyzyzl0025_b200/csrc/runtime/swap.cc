@@ -128,7 +128,13 @@ static void host_dmas(const SlabPool& hp, char* hbase, const Shape& sh, const st
 // (plain st.global to peer addresses) unless BULK is requested explicitly.
 #define ipc_events(flags) (((flags) & AEG_IPC_EVENTS) || (cfg.flags & AEG_CFG_SHARED_HOST))
 
-static int impl_of(const aeg_config& cfg) { return cfg.kernel == AEG_KERNEL_LSU ? IMPL_LSU : IMPL_BULK; }
+// AUTO also picks the warp-broadcast kernel for chunks <= 8 KiB (one chunk per warp iteration).
+static int impl_of(const aeg_config& cfg, uint64_t chunk) {
+  if (cfg.kernel == AEG_KERNEL_LSU) return IMPL_LSU;
+  if (cfg.kernel == AEG_KERNEL_BULK) return IMPL_BULK;
+  if (cfg.kernel == AEG_KERNEL_WARP) return IMPL_WARP;
+  return chunk <= (8u << 10) ? IMPL_WARP : IMPL_BULK;
+}
 
 // ----------------------------------------------------------------------------- swap-out H3
 uint64_t Ctx::swap_out(const Shape& sh, const aeg_block* dev, const aeg_block* host, int32_t n, uint32_t flags) {
@@ -172,7 +178,7 @@ uint64_t Ctx::swap_out(const Shape& sh, const aeg_block* dev, const aeg_block* h
     a.chunk = sh.chunk();
     a.nl = g.lb - g.la;
     a.n = g.i1 - g.i0;
-    launch(0, a, s_gather, impl_of(cfg), 0);
+    launch(0, a, s_gather, impl_of(cfg, sh.chunk()), 0);
     if (tracing)
       tr("op gather gather r=" + cells(0, dp, dev, n, g.la, g.lb, g.i0, g.i1) + " w=" + ring_cells("SO", roff, seg_bytes));
     CUDA_TRY(cudaEventRecord(full, s_gather));
@@ -277,7 +283,7 @@ uint64_t Ctx::swap_in_from(const Shape& sh, int32_t peer, const aeg_block* host,
     a.chunk = sh.chunk();
     a.nl = g.lb - g.la;
     a.n = g.i1 - g.i0;
-    launch(1, a, s_scatter, impl_of(cfg), 0);
+    launch(1, a, s_scatter, impl_of(cfg, sh.chunk()), 0);
     if (tracing)
       tr("op scatter scatter r=" + ring_cells("SI", roff, seg_bytes) + " w=" + cells(0, dp, dev, n, g.la, g.lb, g.i0, g.i1));
     CUDA_TRY(cudaEventRecord(freed, s_scatter));
@@ -348,7 +354,7 @@ uint64_t Ctx::migrate(const Shape& sh, const aeg_block* src, int32_t peer, const
   int32_t lps = 1;
   if (n > 0 && layer < pack) lps = int32_t(std::min<uint64_t>(sh.L, std::max<uint64_t>(1, pack / layer)));
   const int impl = (P && !P->same_process && cfg.kernel == AEG_KERNEL_AUTO) || (P && P->device != device && cfg.kernel == AEG_KERNEL_AUTO)
-                       ? IMPL_LSU : impl_of(cfg);
+                       ? (sh.chunk() <= (8u << 10) ? IMPL_WARP : IMPL_LSU) : impl_of(cfg, sh.chunk());
   for (int32_t la = 0; la < sh.L; la += lps) {
     const int32_t lb = std::min(sh.L, la + lps);
     if (n > 0) {
@@ -393,7 +399,7 @@ uint64_t Ctx::relocate(uint64_t src_off, uint64_t dst_off, uint64_t bytes) {
     CUDA_TRY(cudaEventCreate(&tb));
     CUDA_TRY(cudaEventRecord(ta, s_weights));
   }
-  cudaError_t e = launch_memmove(dev_w, src_off, dst_off, bytes, impl_of(cfg), s_weights, &nl);
+  cudaError_t e = launch_memmove(dev_w, src_off, dst_off, bytes, impl_of(cfg, bytes), s_weights, &nl);
   AEG_REQUIRE(e == cudaSuccess, AEG_ERR_CUDA, "relocate launch failed: %s", cudaGetErrorString(e));
   if (timing) {
     CUDA_TRY(cudaEventRecord(tb, s_weights));

@@ -21,9 +21,15 @@ __global__ void stamp(unsigned long long* t) {
 }
 
 int main() {
-  const uint64_t chunk = 256 << 10;
   const int L = 32;
-  for (int n : {512, 3970}) {
+  struct Case {
+    uint64_t chunk;
+    int n;
+  };
+  for (Case cs : {Case{256 << 10, 512}, Case{256 << 10, 3970}, Case{8 << 10, 16384}, Case{8 << 10, 65536},
+                  Case{2 << 10, 65536}}) {
+    const uint64_t chunk = cs.chunk;
+    const int n = cs.n;
     const uint64_t pool_bytes = uint64_t(n) * chunk * L;
     char *pool, *slot, *hostbuf, *dbuf;
     cudaMalloc(&pool, pool_bytes);
@@ -53,8 +59,8 @@ int main() {
     ca.nl = 1;
     ca.n = n;
     const double alg = 2.0 * n * chunk;
-    for (int impl : {aeg::IMPL_LSU, aeg::IMPL_BULK}) {
-      for (char mode : {'A', 'B', 'C', 'D'}) {
+    for (int impl : {aeg::IMPL_LSU, aeg::IMPL_BULK, aeg::IMPL_WARP}) {
+      for (char mode : {'A', 'C'}) {
         double tot = 0, span = 0;
         const int R = 20;
         for (int r = 0; r < R + 2; ++r) {
@@ -81,9 +87,9 @@ int main() {
             span += (ts[1] - ts[0]) * 1e-6;
           }
         }
-        printf("n=%4d %s %c  event %.1f us (%.0f GB/s)   stamp-to-stamp %.1f us (%.0f GB/s)\n", n,
-               impl == aeg::IMPL_LSU ? "LSU " : "BULK", mode, 1e3 * tot / R, alg / (tot / R) / 1e6, 1e3 * span / R,
-               alg / (span / R) / 1e6);
+        printf("chunk=%6llu n=%5d %s %c  event %.1f us (%.0f GB/s)   stamp-to-stamp %.1f us (%.0f GB/s)\n",
+               (unsigned long long)chunk, n, impl == aeg::IMPL_LSU ? "LSU " : impl == aeg::IMPL_BULK ? "BULK" : "WARP",
+               mode, 1e3 * tot / R, alg / (tot / R) / 1e6, 1e3 * span / R, alg / (span / R) / 1e6);
       }
     }
     cudaFree(pool);
