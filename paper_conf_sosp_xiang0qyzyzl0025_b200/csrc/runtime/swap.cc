@@ -88,6 +88,53 @@ static void host_dmas(const SlabPool& hp, char* hbase, const Shape& sh, const st
                       char* slot, cudaMemcpyKind dir, cudaStream_t s) {
   const uint64_t Cl = sh.chunk(), hstride = hp.lstride(sh);
   const int32_t nseg = g.i1 - g.i0, nl = g.lb - g.la;
+  if (hp.layout == AEG_LAYER_MAJOR && nl == 1) {
+    // One layer: runs of equal length whose host addresses step by a constant pitch (typically whole
+    // slabs: k blocks, pitch S) become ONE 2-D copy — fewer copy-engine commands per layer.
+    size_t q = 0;
+    while (q < runs.size()) {
+      const Run& r0 = runs[q];
+      const int32_t a0 = std::max(r0.i0, g.i0), b0 = std::min(r0.i0 + r0.m, g.i1);
+      if (a0 >= b0) {
+        ++q;
+        continue;
+      }
+      auto host_of = [&](const Run& r, int32_t a) {
+        const aeg_block hb = make_block(AEG_POOL_HOST, block_slab(r.first), block_idx(r.first) + uint32_t(a - r.i0));
+        return hbase + hp.off0(hb, sh) + uint64_t(g.la) * hstride;
+      };
+      char* h0 = host_of(r0, a0);
+      const int32_t m = b0 - a0;
+      size_t e = q + 1;
+      int64_t pitch = 0;
+      char* prev = h0;
+      while (e < runs.size()) {  // extend while the next run is whole, same length, same pitch
+        const Run& r = runs[e];
+        if (r.i0 < g.i0 || r.i0 + r.m > g.i1 || r.m != m || r.i0 != a0 + int32_t(e - q) * m) break;
+        char* cur = host_of(r, r.i0);
+        const int64_t p = cur - prev;
+        if (e == q + 1) pitch = p;
+        if (p != pitch || p < int64_t(m) * int64_t(Cl)) break;
+        prev = cur;
+        ++e;
+      }
+      char* st0 = slot + uint64_t(a0 - g.i0) * Cl;
+      const uint64_t w = uint64_t(m) * Cl;
+      const size_t rows = e - q;
+      if (rows == 1) {
+        if (dir == cudaMemcpyDeviceToHost)
+          CUDA_TRY(cudaMemcpyAsync(h0, st0, w, dir, s));
+        else
+          CUDA_TRY(cudaMemcpyAsync(st0, h0, w, dir, s));
+      } else if (dir == cudaMemcpyDeviceToHost) {
+        CUDA_TRY(cudaMemcpy2DAsync(h0, size_t(pitch), st0, w, w, rows, dir, s));
+      } else {
+        CUDA_TRY(cudaMemcpy2DAsync(st0, w, h0, size_t(pitch), w, rows, dir, s));
+      }
+      q = e;
+    }
+    return;
+  }
   for (const Run& r : runs) {
     const int32_t a = std::max(r.i0, g.i0), b = std::min(r.i0 + r.m, g.i1);
     if (a >= b) continue;
