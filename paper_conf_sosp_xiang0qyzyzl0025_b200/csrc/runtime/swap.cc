@@ -175,12 +175,15 @@ static void host_dmas(const SlabPool& hp, char* hbase, const Shape& sh, const st
 // (plain st.global to peer addresses) unless BULK is requested explicitly.
 #define ipc_events(flags) (((flags) & AEG_IPC_EVENTS) || (cfg.flags & AEG_CFG_SHARED_HOST))
 
-// AUTO also picks the warp-broadcast kernel for chunks <= 8 KiB (one chunk per warp iteration).
+// AUTO by chunk size, from tools/launch_probe.cu (profiles/r01/launch_probe2.txt, TB/s body):
+//   2 KiB chunks: WARP 5.1, LSU 1.7, BULK 0.8     8 KiB: LSU 4.8-5.4, WARP 1.5-4.3, BULK 2.7-2.9
+//   256 KiB: BULK 6.1-6.3, LSU 5.8-6.0
 static int impl_of(const aeg_config& cfg, uint64_t chunk) {
   if (cfg.kernel == AEG_KERNEL_LSU) return IMPL_LSU;
   if (cfg.kernel == AEG_KERNEL_BULK) return IMPL_BULK;
   if (cfg.kernel == AEG_KERNEL_WARP) return IMPL_WARP;
-  return chunk <= (8u << 10) ? IMPL_WARP : IMPL_BULK;
+  if (chunk <= (4u << 10)) return IMPL_WARP;
+  return chunk < (64u << 10) ? IMPL_LSU : IMPL_BULK;
 }
 
 // ----------------------------------------------------------------------------- swap-out H3
@@ -400,8 +403,9 @@ uint64_t Ctx::migrate(const Shape& sh, const aeg_block* src, int32_t peer, const
   const uint64_t layer = uint64_t(n) * sh.chunk();
   int32_t lps = 1;
   if (n > 0 && layer < pack) lps = int32_t(std::min<uint64_t>(sh.L, std::max<uint64_t>(1, pack / layer)));
-  const int impl = (P && !P->same_process && cfg.kernel == AEG_KERNEL_AUTO) || (P && P->device != device && cfg.kernel == AEG_KERNEL_AUTO)
-                       ? (sh.chunk() <= (8u << 10) ? IMPL_WARP : IMPL_LSU) : impl_of(cfg, sh.chunk());
+  // remote pools under AUTO: plain st.global to the peer aperture (LSU / WARP), never bulk copies
+  const int impl = (remote && cfg.kernel == AEG_KERNEL_AUTO) ? (sh.chunk() <= (4u << 10) ? IMPL_WARP : IMPL_LSU)
+                                                             : impl_of(cfg, sh.chunk());
   for (int32_t la = 0; la < sh.L; la += lps) {
     const int32_t lb = std::min(sh.L, la + lps);
     if (n > 0) {
