@@ -111,7 +111,9 @@ typedef struct {
   int32_t kernel;               /* AEG_KERNEL_*                                               */
   int32_t migrate_ctas;         /* CTAs used by the NVLink migrate kernel (SM budget), 0=auto */
   uint32_t flags;               /* AEG_CFG_*                                                  */
-  uint32_t reserved[7];
+  int32_t numa_node;            /* pinned host memory placement: 0 = the GPU's NUMA node (from
+                                   sysfs; unbound if unknown), n > 0 = node n-1, -1 = no binding */
+  uint32_t reserved[6];
 } aeg_config;
 
 /* One checkpoint tensor in the (pageable or registered) host Model Cache, row-major

@@ -29,7 +29,7 @@ namespace aeg {
 enum XferKind { X_SWAP_OUT = 0, X_SWAP_IN, X_MIGRATE, X_WEIGHTS, X_RELOCATE, X_DEBUG, X_IMPORTED };
 
 // Shared (node-wide) CPU KV region: create (exporter) or map (importer), page-locked (engine.cc).
-char* map_shared_host(const std::string& name, uint64_t bytes, bool create);
+char* map_shared_host(const std::string& name, uint64_t bytes, bool create, int numa_node = -1);
 void unmap_shared_host(char* b, uint64_t bytes);
 
 // One transfer: one CUDA event per readiness layer (reading 11) + one completion event.
@@ -131,6 +131,7 @@ struct Ctx {
   char* host_kv = nullptr;
   char* host_stage = nullptr;
   std::string shm_name;   // AEG_CFG_SHARED_HOST: POSIX shm object holding the CPU KV region
+  int numa_bound = -1;    // NUMA node the pinned host memory was bound to (-1: first touch)
   uint64_t host_kv_mapped = 0;
   uint64_t w_bump = 0;
   int w_inflight = 0;
