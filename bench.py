@@ -690,8 +690,11 @@ def migrate_leg_dist(aeg, torch, dist, kernel, n_req=4):
         offs = [OK.addr(geom, sh, h, l) for h in so for l in range(sh.L)]
         keys = [gi.kv_key(1, rank, i, l) for i in range(n) for l in range(sh.L)]
         D.fill_chunks(base, offs, keys, sh.chunk_bytes(), seed)
-    times = []
-    for it in range(5):
+    dst_by_rank = {d: np.array(h, np.uint64) for d, h in enumerate(handles) if h}
+
+    def hand_off(round_pairs):
+        """One timed round: every prefill rank migrates to its partner; the decode side waits per
+        layer on the imported IPC events.  Returns the max-over-ranks device time (ms)."""
         dist.barrier()
         ms = 0.0
         xs = {}
@@ -700,7 +703,7 @@ def migrate_leg_dist(aeg, torch, dist, kernel, n_req=4):
             e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
             e0.record(s)
             ctx.stream_fence(s.cuda_stream)
-            xs = PD.handoff(ctx, sht, src, pairs, rank, {d: np.array(h, np.uint64) for d, h in enumerate(handles) if h})
+            xs = PD.handoff(ctx, sht, src, round_pairs, rank, dst_by_rank)
             for x in xs.values():
                 ctx.layer_ready(x, -1, aeg.READY_WAIT_STREAM, s.cuda_stream)
             e1.record(s)
@@ -716,9 +719,9 @@ def migrate_leg_dist(aeg, torch, dist, kernel, n_req=4):
                     ctx.xfer_release(xi)
         for x in xs.values():
             ctx.xfer_release(x)
-        t = dist.max(ms)
-        if it >= 1:
-            times.append(t)
+        return dist.max(ms)
+
+    times = [hand_off(pairs) for _ in range(5)][1:]
     bad = 0
     if not prefill:
         sender = [s_ for s_, d in pairs if d == rank][0]
@@ -727,13 +730,20 @@ def migrate_leg_dist(aeg, torch, dist, kernel, n_req=4):
         keys = [gi.kv_key(1, sender, i, l) for i in range(n) for l in range(sh.L)]
         bad, _ = D.verify_chunks(base, offs, keys, sh.chunk_bytes(), seed)
     bad = dist.sum(bad)
+    # SURVEY §8(d) C3 for N >= 4: all-to-all, every prefill rank -> every decode rank, round-robin
+    a2a = None
+    if world >= 4:
+        h = world // 2
+        t_rounds = [hand_off(PD.handoff_pairs(world, "all2all", r)) for r in range(h)]
+        a2a = {"rounds": h, "ms_total": round(sum(t_rounds), 3),
+               "GBps_aggregate": round(h * len(pairs) * n * sh.block_bytes() / (sum(t_rounds) * 1e6), 1)}
     ctx.shutdown()
     ms = statistics.median(times)
     payload = len(pairs) * n * sh.block_bytes()
     return {"workload": f"configs[2] Llama-2-13B hand-off, {n_req} requests per pair, pairs {pairs}",
             "payload_bytes": payload, "ms": round(ms, 3), "GBps_aggregate": round(payload / (ms * 1e6), 1),
             "GBps_per_pair": round(payload / len(pairs) / (ms * 1e6), 1), "peak_per_direction_nominal": NVLINK_NOMINAL,
-            "bit_exact": bad == 0}
+            "bit_exact": bad == 0, "all_to_all": a2a}
 
 
 def overlap_leg(aeg, torch, kernel, work_us=500, reps=5):
