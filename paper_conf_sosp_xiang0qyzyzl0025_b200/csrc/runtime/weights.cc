@@ -76,7 +76,8 @@ struct WeightPipe {
   std::condition_variable cv_job, cv_task, cv_filled;
   std::deque<std::unique_ptr<WJob>> jobs;
   std::deque<std::function<void()>> tasks;
-  std::vector<uint8_t> filled;  // per chunk of the current job
+  std::vector<uint8_t> filled;  // per chunk of the current job: parts filled so far
+  static constexpr int kParts = 8;  // fill tasks per chunk (8 MiB each for 64 MiB chunks)
   bool stop = false;
   int nslots = 0;
   uint64_t chunk = 0;
@@ -100,10 +101,14 @@ struct WeightPipe {
   }
 
   // Fill the Stage Buffer slot with the device image of [cs, ce) of job j.
-  void fill(WJob* j, uint64_t ci, int slot, bool wait_slot) {
+  // Fill part `part` of `parts` of chunk ci (the parts of one chunk are queued back to back, so all
+  // threads finish chunk 0 first and its DMA starts after ~1 ms instead of after a whole-chunk copy).
+  void fill(WJob* j, uint64_t ci, int slot, bool wait_slot, int part, int parts) {
     if (wait_slot) cudaEventSynchronize(slot_ev[slot]);  // rule ❸ for the Stage Buffer slot
-    char* dst = c->host_stage + uint64_t(slot) * chunk;
-    const uint64_t cs = j->start + ci * chunk, ce = std::min(j->end, cs + chunk);
+    const uint64_t c0 = j->start + ci * chunk, c1 = std::min(j->end, c0 + chunk);
+    const uint64_t span = (c1 - c0 + parts - 1) / parts;
+    const uint64_t cs = std::min(c1, c0 + span * part), ce = std::min(c1, cs + span);
+    char* dst = c->host_stage + uint64_t(slot) * chunk + (cs - c0);
     uint64_t p = cs;
     auto k0 = std::upper_bound(j->off.begin(), j->off.end(), cs) - j->off.begin();
     for (size_t k = k0 > 0 ? k0 - 1 : 0; k < j->d.size() && j->off[k] < ce; ++k) {
@@ -115,11 +120,12 @@ struct WeightPipe {
       p = b;
     }
     if (ce > p) std::memset(dst + (p - cs), 0, ce - p);
+    bool done;
     {
       std::lock_guard<std::mutex> lk(m);
-      filled[ci] = 1;
+      done = ++filled[ci] == parts;
     }
-    cv_filled.notify_all();
+    if (done) cv_filled.notify_all();
   }
 
   void record_layers(WJob* j, const std::vector<uint64_t>& layer_last, uint64_t upto, cudaStream_t s) {
@@ -194,14 +200,15 @@ struct WeightPipe {
             const uint64_t q = dispatched;
             {
               std::lock_guard<std::mutex> lk(m);
-              tasks.push_back([this, j, q, slot, w] { fill(j, q, slot, w); });
+              for (int part = 0; part < kParts; ++part)
+                tasks.push_back([this, j, q, slot, w, part] { fill(j, q, slot, w, part, kParts); });
             }
-            cv_task.notify_one();
+            cv_task.notify_all();
             ++dispatched;
           }
           {
             std::unique_lock<std::mutex> lk(m);
-            cv_filled.wait(lk, [&] { return filled[ci] != 0; });
+            cv_filled.wait(lk, [&] { return filled[ci] == kParts; });
           }
           const uint64_t cs = j->start + ci * chunk, ce = std::min(j->end, cs + chunk);
           const int slot = slot_of[ci];
