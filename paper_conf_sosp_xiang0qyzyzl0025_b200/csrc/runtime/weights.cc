@@ -31,7 +31,7 @@ uint64_t shard_bytes(const aeg_weight_desc& d, int32_t tp) {
 void copy_shard(char* dst, const aeg_weight_desc& d, int32_t r, int32_t tp, uint64_t a, uint64_t b) {
   const char* src = static_cast<const char*>(d.host_src);
   const uint64_t row = d.cols * uint64_t(d.elem_bytes);
-  if (d.split == AEG_SPLIT_REPLICATED) {
+  if (d.split == AEG_SPLIT_REPLICATED || tp == 1) {  // the shard is the whole, contiguous tensor
     std::memcpy(dst, src + a, b - a);
     return;
   }
@@ -166,7 +166,7 @@ struct WeightPipe {
           char* dst = c->dev_w + j->off[k];
           const char* src = static_cast<const char*>(d.host_src);
           const uint64_t row = d.cols * uint64_t(d.elem_bytes);
-          if (d.split == AEG_SPLIT_REPLICATED) {
+          if (d.split == AEG_SPLIT_REPLICATED || j->tp == 1) {
             CUDA_TRY(cudaMemcpyAsync(dst, src, j->size[k], cudaMemcpyHostToDevice, s));
           } else if (d.split == AEG_SPLIT_ROW) {
             const uint64_t w = row / uint64_t(j->tp);
