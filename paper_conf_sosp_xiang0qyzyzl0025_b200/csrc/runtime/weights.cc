@@ -28,31 +28,14 @@ uint64_t shard_bytes(const aeg_weight_desc& d, int32_t tp) {
   return d.split == AEG_SPLIT_REPLICATED ? all : all / uint64_t(tp);
 }
 
-// Host copy granularity of contiguous shard bytes (0 = one memcpy per range); AEG_FILL_PIECE env
-// override for measurements.
-uint64_t fill_piece() {
-  static const uint64_t v = [] {
-    const char* e = std::getenv("AEG_FILL_PIECE");
-    return e ? uint64_t(std::strtoull(e, nullptr, 10)) : uint64_t(0);
-  }();
-  return v;
-}
-
-void copy_contig(char* dst, const char* src, uint64_t n) {
-  const uint64_t p = fill_piece();
-  if (!p) {
-    std::memcpy(dst, src, n);
-    return;
-  }
-  for (uint64_t o = 0; o < n; o += p) std::memcpy(dst + o, src + o, std::min(p, n - o));
-}
-
-// Copy bytes [a, b) of rank r's shard of tensor d into dst (Megatron splits, reading 18).
+// Copy bytes [a, b) of rank r's shard of tensor d into dst (Megatron splits, reading 18).  The copy
+// granularity of contiguous ranges was swept (16 KiB .. one memcpy per range): no measurable effect
+// on the staged switch (profiles/r01/sweep3).
 void copy_shard(char* dst, const aeg_weight_desc& d, int32_t r, int32_t tp, uint64_t a, uint64_t b) {
   const char* src = static_cast<const char*>(d.host_src);
   const uint64_t row = d.cols * uint64_t(d.elem_bytes);
   if (d.split == AEG_SPLIT_REPLICATED || tp == 1) {  // the shard is the whole, contiguous tensor
-    copy_contig(dst, src + a, b - a);
+    std::memcpy(dst, src + a, b - a);
     return;
   }
   if (d.split == AEG_SPLIT_COL || d.split == AEG_SPLIT_VOCAB) {
