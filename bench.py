@@ -572,6 +572,7 @@ def switch_leg(aeg, torch, n_switch, kernel, descs, mode="staged", caches=None):
             pre = (nn, xp, int(o[0]))
     if pre is not None:
         ctx.layer_ready(pre[1], -1, aeg.READY_BLOCK)
+    wchunks, wfill, wslot = ctx.weights_stats()
     ctx.shutdown()
     per = {}
     for nm in names:
@@ -593,7 +594,9 @@ def switch_leg(aeg, torch, n_switch, kernel, descs, mode="staged", caches=None):
            "prefetch": "weights prefetched during the previous turn, relocated on-device at the switch (3.b)"}[mode]
     return {"workload": f"configs[3] 3-model switch (Qwen-1.8B, Llama-7B, Yi-9B shapes), 1 GiB KV each; {how}",
             "per_model": per, "weights_bit_exact_sample": bad == 0, "register_s": reg_s,
-            "landing_ms_one_switch": diag_ms}
+            "landing_ms_one_switch": diag_ms,
+            "weight_pipeline": {"chunks": wchunks, "issuer_wait_fill_ms": round(wfill, 1),
+                                "fill_wait_slot_ms": round(wslot, 1)}}
 
 
 def migrate_leg(aeg, torch, kernel, n_req=4):

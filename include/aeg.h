@@ -294,6 +294,11 @@ int aeg_weights_region(aeg_ctx ctx, void** base, uint64_t* bytes, uint64_t* bump
 int aeg_weights_relocate(aeg_ctx ctx, uint64_t src_off, uint64_t dst_off, uint64_t bytes,
                          aeg_xfer* out);
 
+/* Weight-pipeline counters since init: chunks issued, host milliseconds the issuer waited for host
+ * fills (fill-bound), and summed milliseconds fill tasks waited for a Stage Buffer slot's previous
+ * DMA (PCIe-bound).  Any output pointer may be NULL. */
+int aeg_weights_stats(aeg_ctx ctx, uint64_t* chunks, double* issuer_wait_fill_ms, double* fill_wait_slot_ms);
+
 /* Page-lock an existing host range (e.g. a Model Cache) so weights in it DMA directly. */
 int aeg_host_register(aeg_ctx ctx, void* ptr, uint64_t bytes);
 int aeg_host_unregister(aeg_ctx ctx, void* ptr);

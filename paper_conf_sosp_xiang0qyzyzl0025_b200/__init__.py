@@ -111,6 +111,7 @@ _SIGS = {
     "aeg_weights_reset": [P, U64],
     "aeg_weights_region": [P, C.POINTER(P), PU64, PU64],
     "aeg_weights_relocate": [P, U64, U64, U64, PU64],
+    "aeg_weights_stats": [P, PU64, C.POINTER(C.c_double), C.POINTER(C.c_double)],
     "aeg_host_register": [P, P, U64],
     "aeg_host_unregister": [P, P],
     "aeg_export_ipc": [P, P, PU64],
@@ -315,6 +316,12 @@ class Context:
         x = C.c_uint64()
         _chk(lib().aeg_weights_relocate(self.h, int(src_off), int(dst_off), int(nbytes), C.byref(x)))
         return x.value
+
+    def weights_stats(self):
+        """(chunks issued, issuer ms waiting for host fills, fill ms waiting for Stage Buffer slots)."""
+        n, a, b = C.c_uint64(), C.c_double(), C.c_double()
+        _chk(lib().aeg_weights_stats(self.h, C.byref(n), C.byref(a), C.byref(b)))
+        return n.value, a.value, b.value
 
     def host_register(self, ptr: int, nbytes: int):
         _chk(lib().aeg_host_register(self.h, P(ptr), int(nbytes)))

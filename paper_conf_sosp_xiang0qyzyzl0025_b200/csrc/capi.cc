@@ -404,6 +404,14 @@ int aeg_weights_relocate(aeg_ctx ctx, uint64_t src_off, uint64_t dst_off, uint64
   });
 }
 
+int aeg_weights_stats(aeg_ctx ctx, uint64_t* chunks, double* issuer_wait_fill_ms, double* fill_wait_slot_ms) {
+  return guarded([&] {
+    Ctx& c = C(ctx);
+    c.weights_counters(chunks, issuer_wait_fill_ms, fill_wait_slot_ms);
+    return AEG_OK;
+  });
+}
+
 int aeg_host_register(aeg_ctx ctx, void* ptr, uint64_t bytes) {
   return guarded([&] {
     Ctx& c = C(ctx);

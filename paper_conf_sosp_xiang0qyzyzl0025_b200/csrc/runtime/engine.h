@@ -212,6 +212,7 @@ struct Ctx {
   uint64_t weights_stage(const aeg_weight_desc* d, int32_t n, int32_t r, int32_t tp, uint64_t* offs);
   void weights_start();
   void weights_stop();
+  void weights_counters(uint64_t* chunks, double* wait_fill_ms, double* wait_slot_ms);
 };
 
 }  // namespace aeg

@@ -11,6 +11,7 @@
 // When every tensor lies in host memory registered with aeg_host_register the workers are skipped
 // and the issuer DMAs shards straight from the Model Cache (2-D copies for ROW shards).
 #include <algorithm>
+#include <chrono>
 #include <condition_variable>
 #include <cstdlib>
 #include <cstring>
@@ -87,6 +88,15 @@ struct WeightPipe {
   uint64_t next_slot = 0;
   std::vector<cudaEvent_t> slot_ev;
   std::vector<uint8_t> slot_used;
+  // counters (aeg_weights_stats)
+  std::atomic<uint64_t> n_chunks{0};
+  std::atomic<uint64_t> wait_fill_ns{0}, wait_slot_ns{0};
+
+  static uint64_t now_ns() {
+    return uint64_t(std::chrono::duration_cast<std::chrono::nanoseconds>(
+                        std::chrono::steady_clock::now().time_since_epoch())
+                        .count());
+  }
 
   void worker_loop() {
     cudaSetDevice(c->device);
@@ -107,7 +117,11 @@ struct WeightPipe {
   // Fill part `part` of `parts` of chunk ci (the parts of one chunk are queued back to back, so all
   // threads finish chunk 0 first and its DMA starts after ~1 ms instead of after a whole-chunk copy).
   void fill(WJob* j, uint64_t ci, int slot, bool wait_slot, int part, int parts) {
-    if (wait_slot) cudaEventSynchronize(slot_ev[slot]);  // rule ❸ for the Stage Buffer slot
+    if (wait_slot) {  // rule ❸ for the Stage Buffer slot
+      const uint64_t t0 = now_ns();
+      cudaEventSynchronize(slot_ev[slot]);
+      wait_slot_ns += now_ns() - t0;
+    }
     const uint64_t c0 = j->start + ci * chunk, c1 = std::min(j->end, c0 + chunk);
     const uint64_t span = (c1 - c0 + parts - 1) / parts;
     const uint64_t cs = std::min(c1, c0 + span * part), ce = std::min(c1, cs + span);
@@ -210,9 +224,12 @@ struct WeightPipe {
             ++dispatched;
           }
           {
+            const uint64_t t0 = now_ns();
             std::unique_lock<std::mutex> lk(m);
             cv_filled.wait(lk, [&] { return filled[ci] == kParts; });
+            wait_fill_ns += now_ns() - t0;
           }
+          n_chunks++;
           const uint64_t cs = j->start + ci * chunk, ce = std::min(j->end, cs + chunk);
           const int slot = slot_of[ci];
           CUDA_TRY(cudaMemcpyAsync(c->dev_w + cs, c->host_stage + uint64_t(slot) * chunk, ce - cs,
@@ -259,6 +276,12 @@ struct WeightPipe {
 
 Ctx::Ctx() = default;
 Ctx::~Ctx() = default;
+
+void Ctx::weights_counters(uint64_t* chunks, double* wait_fill_ms, double* wait_slot_ms) {
+  if (chunks) *chunks = wp ? wp->n_chunks.load() : 0;
+  if (wait_fill_ms) *wait_fill_ms = wp ? wp->wait_fill_ns.load() * 1e-6 : 0.0;
+  if (wait_slot_ms) *wait_slot_ms = wp ? wp->wait_slot_ns.load() * 1e-6 : 0.0;
+}
 
 void Ctx::weights_start() {
   wp = std::make_unique<WeightPipe>();
