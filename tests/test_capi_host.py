@@ -197,6 +197,36 @@ def test_block_offsets_match_oracle_addr(layout):
     c.shutdown()
 
 
+def test_block_offsets_errors_stats_peaks_and_free_after():
+    c = host_ctx(3)
+    try:
+        a = c.kv_alloc(0, A, 3)
+        with pytest.raises(aeg.AegError) as e:
+            c.block_offsets(0, Bs, a)                     # another shape
+        assert e.value.code == aeg.ERR_INVALID
+        b = c.kv_alloc(0, Bs, 1)
+        c.kv_free(0, b)
+        with pytest.raises(aeg.AegError) as e:
+            c.block_offsets(0, A, [a[0], b[0]])           # b is no longer owned (slab reclaimed)
+        assert e.value.code in (aeg.ERR_STATE, aeg.ERR_INVALID)
+        s = c.stats(0)
+        assert s.peak_used_bytes >= s.used_bytes and s.peak_assigned_bytes >= s.assigned_bytes
+        assert s.peak_assigned_bytes == 3 * SLAB             # A used 2 slabs, Bs one more at the peak
+        # aeg_kv_free_after: blocks stay in the move list until the named transfer completes (❸)
+        x = c.debug_xfer_begin(0, a[:1])
+        c.kv_free_after(0, a, x)
+        assert c.stats(0).quarantined_blocks == 3
+        c.reclaim()
+        assert c.stats(0).quarantined_blocks == 3
+        c.debug_xfer_complete(x)
+        c.reclaim()
+        s = c.stats(0)
+        assert s.quarantined_blocks == 0 and s.free_slabs == 3
+        assert aeg.default_config().numa_node == 0           # default: the GPU's NUMA node
+    finally:
+        c.shutdown()
+
+
 def test_daemon_reclaims_move_list():
     """With the daemon running, a move-list block is reclaimed without an explicit aeg_reclaim."""
     import time
