@@ -256,4 +256,25 @@ int aegin_host_fill(void* p, uint64_t nbytes, uint64_t seed, uint64_t key, int t
   return 0;
 }
 
+// Strided variant: `rows` runs of `width` bytes at a `pitch`, run r starting at p + r * pitch; every
+// word holds the value it has in the dense fill of the whole [rows x pitch] region with base `key`,
+// so a run is bit-identical to the same bytes of a dense fill (used to materialise only one TP
+// rank's column slice of a row-major tensor in a sparse Model Cache).  pitch, width multiples of 8.
+int aegin_host_fill_2d(void* p, uint64_t rows, uint64_t pitch, uint64_t width, uint64_t seed, uint64_t key,
+                       int threads) {
+  if ((pitch & 7) || (width & 7) || width > pitch) return 1;
+  if (threads < 1) threads = 1;
+  std::vector<std::thread> ts;
+  for (int t = 0; t < threads; ++t)
+    ts.emplace_back([=] {
+      for (uint64_t r = rows * t / threads; r < rows * (t + 1) / threads; ++r) {
+        uint64_t* q = reinterpret_cast<uint64_t*>(static_cast<char*>(p) + r * pitch);
+        const uint64_t w0 = r * pitch / 8;
+        for (uint64_t w = 0; w < width / 8; ++w) q[w] = sm64(seed ^ (key + w0 + w));
+      }
+    });
+  for (auto& t : ts) t.join();
+  return 0;
+}
+
 }  // extern "C"

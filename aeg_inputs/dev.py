@@ -32,6 +32,7 @@ def lib():
             "aegin_copy": [P, P, U64],
             "aegin_sync": [],
             "aegin_host_fill": [P, U64, U64, U64, C.c_int],
+            "aegin_host_fill_2d": [P, U64, U64, U64, U64, U64, C.c_int],
         }
         for k, a in sig.items():
             getattr(L, k).argtypes = a
@@ -120,3 +121,9 @@ def write(ptr: int, arr: np.ndarray):
 
 def host_fill(arr: np.ndarray, seed: int, key: int, threads: int = 8):
     _ck(lib().aegin_host_fill(P(arr.ctypes.data), arr.nbytes, seed, key, threads))
+
+
+def host_fill_2d(ptr: int, rows: int, pitch: int, width: int, seed: int, key: int, threads: int = 8):
+    """Fill `rows` runs of `width` bytes at `pitch` from `ptr` with the bytes a dense host_fill of
+    the [rows x pitch] region (key base `key`) would put there."""
+    _ck(lib().aegin_host_fill_2d(P(ptr), rows, pitch, width, seed, key, threads))

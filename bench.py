@@ -59,6 +59,7 @@ def parse():
     p.add_argument("--kernel", default="auto", choices=["auto", "lsu", "bulk"])
     p.add_argument("--no-switch", action="store_true")
     p.add_argument("--no-migrate", action="store_true")
+    p.add_argument("--no-c5", action="store_true", help="skip the configs[4] Qwen-72B TP=4 scale-up leg")
     p.add_argument("--no-e2e", action="store_true")
     p.add_argument("--no-cpu", action="store_true")
     p.add_argument("--switches", type=int, default=30)
@@ -181,13 +182,16 @@ def peaks():
     return HBM_FALLBACK, "fallback"
 
 
-def ncu_traffic(kind: str):
-    """Per-launch dram bytes of our kernel from the committed ncu --set full summary, if any."""
+def ncu_traffic(kind: str, alg_bytes_per_launch: int):
+    """Per-launch DRAM bytes (read + write) of our kernel from the committed ncu capture of the same
+    launch (profiles/ncu_summary.json), or None when that capture was of a different launch size."""
     p = os.path.join(ROOT, "profiles", "ncu_summary.json")
     if not os.path.exists(p):
         return None
-    d = json.load(open(p))
-    return d.get(kind, {}).get("dram_bytes_per_launch")
+    d = json.load(open(p)).get(kind, {})
+    if int(d.get("algorithmic_bytes_per_launch", -1)) != int(alg_bytes_per_launch):
+        return None
+    return d.get("dram_bytes_per_launch")
 
 
 # ----------------------------------------------------------------------------------- workload
@@ -749,6 +753,205 @@ def migrate_leg_dist(aeg, torch, dist, kernel, n_req=4):
             "bit_exact": bad == 0, "all_to_all": a2a}
 
 
+def sparse_model_cache(name, m, tp_rank, tp_size, seed, threads=16, min_sparse=MIB):
+    """Host Model Cache of a whole model (pageable) laid out as model_caches()
+    does, but only TP rank `tp_rank`'s shard bytes are materialised: the rest of the anonymous
+    MAP_NORESERVE mapping is never touched, so a 144.6 GB Qwen-72B cache costs one rank's 36 GB of
+    host RAM.  Materialised bytes equal the dense content (the generator is counter-based)."""
+    import mmap
+    import aeg_inputs as gi
+    from aeg_inputs import dev as D
+    ts = gi.model_tensors(name)
+    sizes = [t["rows"] * t["cols"] * 2 for t in ts]
+    offs = np.cumsum([0] + [-(-x // 256) * 256 for x in sizes])
+    mm = mmap.mmap(-1, int(offs[-1]), flags=mmap.MAP_PRIVATE | mmap.MAP_ANONYMOUS | getattr(mmap, "MAP_NORESERVE", 0x4000))
+    if hasattr(mmap, "MADV_NOHUGEPAGE"):
+        mm.madvise(mmap.MADV_NOHUGEPAGE)
+    buf = np.frombuffer(mm, dtype=np.uint8)
+    base = buf.ctypes.data
+    touched = 0
+    for k, (t, o, n) in enumerate(zip(ts, offs, sizes)):
+        o, rb, key = int(o), t["cols"] * 2, gi.weight_key(m, k)
+        if t["split"] == gi.REPLICATED or n < min_sparse or tp_size == 1:
+            D.host_fill(buf[o:o + n], seed, key, threads=threads)
+            touched += n
+        elif t["split"] in (gi.COL, gi.VOCAB):
+            g_rows = t["rows"] // t["groups"]
+            part = g_rows // tp_size
+            for g in range(t["groups"]):
+                a = (g * g_rows + tp_rank * part) * rb
+                assert a % 8 == 0
+                D.host_fill(buf[o + a:o + a + part * rb], seed, key + a // 8, threads=threads)
+                touched += part * rb
+        else:   # ROW: the rank's column slice of every row
+            w = rb // tp_size
+            D.host_fill_2d(base + o + tp_rank * w, t["rows"], rb, w, seed, key + tp_rank * w // 8, threads=threads)
+            touched += t["rows"] * w
+    descs = [dict(host_src=base + int(o), rows=t["rows"], cols=t["cols"], elem_bytes=2, layer=t["layer"],
+                  split=t["split"], groups=t["groups"]) for t, o in zip(ts, offs)]
+    return descs, (mm, buf), touched
+
+
+def _c5_check_weights(aeg, ctx, name, m, seed, tp_rank, tp_size, got_offs, picks):
+    """Sampled O8 parity: the oracle shards the densely generated tensor; the device copy must match."""
+    import aeg_inputs as gi
+    from aeg_inputs import dev as D
+    from oracle import weights as W
+    ts = gi.model_tensors(name)
+    shard_sizes = [t["rows"] * t["cols"] * 2 // (1 if t["split"] == W.REPLICATED else tp_size) for t in ts]
+    exp_offs, _ = W.bump_offsets(shard_sizes, 0)
+    ok = [int(o) for o in got_offs] == exp_offs
+    base, _, _ = ctx.weights_region()
+    bad = 0
+    for k in picks:
+        t = ts[k]
+        full = gi.region_bytes(seed, gi.weight_key(m, k), t["rows"] * t["cols"] * 2).reshape(t["rows"], t["cols"], 2)
+        exp = np.ascontiguousarray(W.shard(full, t["split"], t["groups"], tp_rank, tp_size)).reshape(-1)
+        bad += int((D.read(base + exp_offs[k], exp.size) != exp).sum())
+    return ok and bad == 0, len(picks)
+
+
+def c5_leg(aeg, torch, kernel, dist=None, tp_rank=1, tp_size=4, reps=3):
+    """configs[4]: Qwen-72B TP=4 scale-up.  The decode instance's rank r stages its 36.1 GB weight
+    shard (Megatron col/row/vocab split, host threads -> pinned Stage Buffer -> PCIe, PAPER.md:
+    1343-1354) while its prefill partner hands it 2 GiB of KV (Qwen-72B-TP4 shape, H=16 per rank)
+    through the fused migrate kernel (PAPER.md:2096-2098 layout).  One GPU: one rank pair, the
+    prefill side a second context on the same GPU (the same kernel stores over NVLink when the peer
+    is another GPU); with 8 ranks: ranks 0-3 prefill, 4-7 decode, rank i -> i + 4.
+    Reports per-rank weights GB/s, KV hand-off GB/s and the scale-up time (both ready)."""
+    import aeg_inputs as gi
+    from aeg_inputs import dev as D
+    from oracle import kv as OK
+    from oracle.shape import KVShape
+    world = 1 if dist is None else dist.world
+    rank = 0 if dist is None else dist.rank
+    device = 0 if dist is None else dist.device
+    decode = world == 1 or rank >= world // 2
+    prefill = world == 1 or rank < world // 2
+    if world > 1:
+        tp_rank = rank % (world // 2)
+    seed_w, seed_kv = gi.w_seed(5), gi.kv_seed(5)
+    sht = gi.KV_SHAPES["qwen-72b-tp4"]
+    sh = KVShape(*sht)
+    n_kv = (2 * GIB) // sh.block_bytes()
+    slab = 10 * 64 * MIB * 2            # 1.25 GiB: 128 blocks of 10 MiB
+    nslab = -(-n_kv // (slab // sh.block_bytes())) + 1
+    out = {"workload": "configs[4] Qwen-72B TP=4 scale-up: one decode rank stages its weight shard (staged 3.a) "
+                       f"while its prefill partner migrates {n_kv} blocks ({n_kv * sh.block_bytes() / GIB:.2f} GiB) "
+                       "of KV to it" + (" (1 GPU: both ranks' contexts on it)" if world == 1 else f", {world} ranks")}
+    descs, keep, touched, wctx, a, b = None, None, 0, None, None, None
+    t0 = time.time()
+    if decode:
+        descs, keep, touched = sparse_model_cache("qwen-72b", 7, tp_rank, tp_size, seed_w)
+        shard_total = sum(-(-(d["rows"] * d["cols"] * 2 // (1 if d["split"] == gi.REPLICATED else tp_size)) // 256) * 256
+                          for d in descs)
+        wctx = aeg.Context(device, aeg.default_config(device_kv_bytes=nslab * slab, host_kv_bytes=GIB,
+                                                      dev_slab_bytes=slab, dev_slab_layout=aeg.BLOCK_MAJOR,
+                                                      device_weight_bytes=shard_total + 64 * MIB, kernel=kernel,
+                                                      host_threads=12, flags=aeg.CFG_TIMING))
+        b = wctx
+    out["model_cache_build_s"] = round(time.time() - t0, 1)
+    out["model_cache_touched_bytes"] = touched
+    if prefill:
+        a = aeg.Context(device, aeg.default_config(device_kv_bytes=nslab * slab, host_kv_bytes=GIB, dev_slab_bytes=slab,
+                                                   dev_slab_layout=aeg.LAYER_MAJOR, kernel=kernel, flags=aeg.CFG_TIMING))
+    geom_a = OK.PoolGeom(nslab * slab, slab, aeg.LAYER_MAJOR)
+    geom_b = OK.PoolGeom(nslab * slab, slab, aeg.BLOCK_MAJOR)
+    # pools + destination handles
+    if world == 1:
+        a.import_peer(1, b.export_ipc())
+        peer_of = {0: 1}
+        dst = b.kv_alloc(0, sht, n_kv)
+    else:
+        from paper_conf_sosp_xiang0qyzyzl0025_b200 import dist as PD
+        ctx = a if prefill else b
+        PD.connect(ctx, rank)
+        dst = None if prefill else b.kv_alloc(0, sht, n_kv)
+        handles = PD.exchange(None if prefill else [int(x) for x in dst])
+        peer_of = {rank: rank + world // 2} if prefill else {}
+        dst_by_rank = {d: np.array(h, np.uint64) for d, h in enumerate(handles) if h}
+    src = None
+    if prefill:
+        src = a.kv_alloc(0, sht, n_kv)
+        abase, _ = a.pool_region(0)
+        so = [aeg.decode_block(x)[1:] for x in src]
+        D.fill_chunks(abase, [OK.addr(geom_a, sh, h, l) for h in so for l in range(sh.L)],
+                      [gi.kv_key(5, rank, i, l) for i in range(n_kv) for l in range(sh.L)], sh.chunk_bytes(), seed_kv)
+    dst_handles = dst if world == 1 else (dst_by_rank.get(rank + world // 2) if prefill else None)
+    D.sync()
+
+    def one(do_w, do_kv):
+        if dist is not None:
+            dist.barrier()
+        s = torch.cuda.Stream()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(s)
+        xw = xk = None
+        if decode and do_w:
+            b.stream_fence(s.cuda_stream)
+            b.weights_reset(0)
+            offs, xw = b.weights_stage(descs, tp_rank, tp_size)
+        if prefill and do_kv:
+            a.stream_fence(s.cuda_stream)
+            xk = a.kv_migrate(sht, src, peer_of[rank], dst_handles)
+        if xw is not None:
+            b.layer_ready(xw, -1, aeg.READY_WAIT_STREAM, s.cuda_stream)
+        if xk is not None:
+            a.layer_ready(xk, -1, aeg.READY_WAIT_STREAM, s.cuda_stream)
+        e1.record(s)
+        e1.synchronize()
+        ms = e0.elapsed_time(e1) if (xw is not None or xk is not None) else 0.0
+        if xw is not None:
+            b.xfer_release(xw)
+        if xk is not None:
+            a.xfer_release(xk)
+        return ms if dist is None else dist.max(ms)
+
+    w_ms = [one(True, False) for _ in range(reps)]
+    k_ms = [one(False, True) for _ in range(reps + 2)][2:]
+    both = [one(True, True) for _ in range(reps)]
+    w_ok, picks = True, 0
+    if decode:
+        n_t = len(descs)
+        pick = [0, 1, 2, 3, 4, 5, 6, 7, n_t // 2 + 3, n_t - 2]
+        b.weights_reset(0)
+        offs, x = b.weights_stage(descs, tp_rank, tp_size)
+        b.layer_ready(x, -1, aeg.READY_BLOCK)
+        b.xfer_release(x)
+        w_ok, picks = _c5_check_weights(aeg, b, "qwen-72b", 7, seed_w, tp_rank, tp_size, offs, pick)
+    kv_bad = 0
+    if decode:
+        sender = 0 if world == 1 else rank - world // 2
+        bbase, _ = b.pool_region(0)
+        do = [aeg.decode_block(x)[1:] for x in dst]
+        kv_bad, _ = D.verify_chunks(bbase, [OK.addr(geom_b, sh, h, l) for h in do for l in range(sh.L)],
+                                    [gi.kv_key(5, sender, i, l) for i in range(n_kv) for l in range(sh.L)],
+                                    sh.chunk_bytes(), seed_kv)
+    shard = 0 if not decode else sum(d["rows"] * d["cols"] * 2 // (1 if d["split"] == gi.REPLICATED else tp_size)
+                                     for d in descs)
+    for c in (a, b):
+        if c is not None:
+            c.shutdown()
+    del keep
+    n_dec = 1 if world == 1 else world // 2
+    if dist is not None:
+        shard = dist.max(shard)
+        kv_bad = dist.sum(kv_bad)
+        w_ok = dist.sum(0 if w_ok else 1) == 0
+    kvb = n_kv * sh.block_bytes()
+    wm, km, bm = statistics.median(w_ms), statistics.median(k_ms), statistics.median(both)
+    out.update({"tp_size": tp_size, "decode_ranks": n_dec, "shard_bytes_per_rank": int(shard),
+                "weights_ms": round(wm, 1), "weights_GBps_per_rank": round(shard / (wm * 1e6), 1),
+                "weights_frac_of_pcie_nominal": round(shard / (wm * 1e6) / PCIE_NOMINAL, 3),
+                "kv_bytes_per_pair": kvb, "kv_ms": round(km, 3), "kv_GBps_per_pair": round(kvb / (km * 1e6), 1),
+                "kv_peer": "same GPU (HBM)" if world == 1 else "NVLink",
+                "scale_up_ms": round(bm, 1), "scale_up_ms_all": [round(x, 1) for x in both],
+                "aggregate_h2d_GBps": round(n_dec * shard / (bm * 1e6), 1),
+                "weights_bit_exact_sample": bool(w_ok), "weights_tensors_checked": picks,
+                "kv_bit_exact": kv_bad == 0})
+    return out
+
+
 def overlap_leg(aeg, torch, kernel, work_us=500, reps=5):
     """North star: "decoding of layer i overlaps the transfer of layer i+1".  A 1 GiB Llama-7B KV
     batch (32 layers) is swapped in while a synthetic decode step does `work_us` of work per layer
@@ -944,9 +1147,16 @@ def run_ours(args):
                   "model_cache_gen_s": round(gen_s, 1)}
             del caches
         ovl = None if args.no_switch or world > 1 else overlap_leg(aeg, torch, kernel)
+        if args.no_c5:
+            c5 = None
+        elif world in (1, 8):
+            c5 = c5_leg(aeg, torch, kernel, dist if world > 1 else None)
+        else:
+            c5 = {"skipped": "configs[4] is the 8-GPU TP=4 layout (one rank pair on 1 GPU); not defined for N=%d" % world}
         cpu = None if args.no_cpu or rank != 0 else cpu_baseline()
         out.update({"e2e": e2e, "verify": ver, "one_direction": one_dir, "pcie_memcpy_GBps": {k: round(v, 1) for k, v in pc.items()},
-                    "switch": sw, "migrate": mig, "per_layer_overlap": ovl, "cpu_baseline": cpu})
+                    "switch": sw, "migrate": mig, "per_layer_overlap": ovl, "c5": c5,
+                    "cpu_baseline": cpu})
         if not ver["ok"]:
             log("VERIFICATION FAILED", ver)
     else:
@@ -965,7 +1175,7 @@ def run_ours(args):
                        "staging_slots": sb.cfg.staging_slots, "parallelism": f"replicas x{world}"},
             "roofline": {"bound": "hbm", "kernel": "gather (swap-out, H2)", "achieved": round(g_ach, 1),
                          "peak": hbm, "peak_source": hbm_src, "unit": "GB/s",
-                         "frac": round(g_ach / hbm, 3), "traffic": ncu_traffic("gather"),
+                         "frac": round(g_ach / hbm, 3), "traffic": ncu_traffic("gather", int(g_per_launch_bytes)),
                          "algorithmic_bytes_per_launch": int(g_per_launch_bytes), "launches": g[0],
                          "mean_launch_ms": round(g_ms, 4), "scatter_achieved": round(s_ach, 1)},
             "pcie": {"bound": "pcie", "achieved_round_trip": round(bytes_step / (ms_step * 1e6), 1),

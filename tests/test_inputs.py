@@ -47,3 +47,39 @@ def test_churn_ops_shape():
     frees = [o for o in ops if o[0] == "free"]
     assert sum(n for _, n in allocs) <= 900
     assert len(frees) == len(allocs) // 2
+
+
+def test_host_fill_matches_numpy_and_2d_matches_dense():
+    from aeg_inputs import dev as D
+    dense = np.zeros(64 * 48, dtype=np.uint8)
+    D.host_fill(dense, 9, 1234, threads=3)
+    assert np.array_equal(dense, gi.region_bytes(9, 1234, dense.size))
+    part = np.zeros_like(dense)
+    D.host_fill_2d(part.ctypes.data + 16, 64, 48, 24, 9, 1234 + 2, threads=4)
+    m = np.zeros((64, 48), bool)
+    m[:, 16:40] = True
+    assert np.array_equal(part.reshape(64, 48)[m], dense.reshape(64, 48)[m])
+    assert not part.reshape(64, 48)[~m].any()
+
+
+def test_sparse_model_cache_materialises_exactly_one_shard():
+    """bench.sparse_model_cache (configs[4] host cache): rank r's shard bytes equal the dense cache's,
+    every other byte is untouched (zero), checked through the oracle's shard rule (O8)."""
+    import bench
+    from oracle import weights as W
+    dense_descs, dense_caches = bench.model_caches(["tiny"])
+    dense = dense_caches["tiny"]
+    for r in range(2):
+        descs, keep, touched = bench.sparse_model_cache("tiny", 0, r, 2, gi.w_seed(3), min_sparse=0)
+        buf = keep[1]
+        assert buf.size == dense.size
+        tot = 0
+        for d, dd in zip(descs, dense_descs["tiny"]):
+            o = d["host_src"] - buf.ctypes.data
+            n = d["rows"] * d["cols"] * 2
+            got = buf[o:o + n].reshape(d["rows"], d["cols"], 2)
+            exp = dense[o:o + n].reshape(d["rows"], d["cols"], 2)
+            gs = W.shard(got, d["split"], d["groups"], r, 2)
+            assert np.array_equal(gs, W.shard(exp, d["split"], d["groups"], r, 2))
+            tot += gs.size
+        assert int(np.count_nonzero(buf)) <= tot == touched

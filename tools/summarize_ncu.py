@@ -73,5 +73,39 @@ def main(d):
     print(json.dumps(summ, indent=1))
 
 
+def fullsize(csv_path, alg_bytes, capture):
+    """Merge a single-pass launch list (gpu__time_duration + dram__bytes_{read,write}, one row per
+    metric) of the bench's own full-size step into profiles/ncu_summary.json under gather/scatter:
+    per-launch DRAM traffic next to the algorithmic bytes of the same launch (bench.py roofline)."""
+    txt = open(csv_path).read()
+    rows = list(csv.DictReader(io.StringIO(txt[txt.index('"ID"'):])))
+    by = collections.defaultdict(lambda: collections.defaultdict(list))
+    names = {}
+    for r in rows:
+        ro = role(r["Kernel Name"])
+        if ro:
+            by[ro][r["Metric Name"]].append(float(r["Metric Value"].replace(",", "")))
+            names[ro] = r["Kernel Name"].split("::")[-1][:60] + f" grid {r['Grid Size']} block {r['Block Size']}"
+    out_p = os.path.join(os.path.dirname(os.path.dirname(os.path.abspath(__file__))), "profiles", "ncu_summary.json")
+    summ = json.load(open(out_p)) if os.path.exists(out_p) else {}
+    for ro, m in by.items():
+        n = len(m["gpu__time_duration.sum"])
+        rd, wr = sum(m["dram__bytes_read.sum"]) / n, sum(m["dram__bytes_write.sum"]) / n
+        dur = sum(m["gpu__time_duration.sum"]) / n
+        if ro in summ and "16" in summ[ro].get("capture", ""):
+            summ[ro + "_set_full_16req"] = summ.pop(ro)
+        summ[ro] = {"kernel": names[ro], "capture": capture, "launches": n,
+                    "algorithmic_bytes_per_launch": int(alg_bytes),
+                    "dram_bytes_per_launch": int(rd + wr), "dram_read_bytes_per_launch": int(rd),
+                    "dram_write_bytes_per_launch": int(wr), "duration_us_cold_serialised": round(dur / 1e3, 2),
+                    "algorithmic_GBps_cold_serialised": round(alg_bytes / dur, 1),
+                    "traffic_over_algorithmic": round((rd + wr) / alg_bytes, 4)}
+    json.dump(summ, open(out_p, "w"), indent=1)
+    print(json.dumps(summ, indent=1))
+
+
 if __name__ == "__main__":
-    main(sys.argv[1] if len(sys.argv) > 1 else "gpurun_out/ncu_final")
+    if len(sys.argv) > 1 and sys.argv[1] == "--fullsize":
+        fullsize(sys.argv[2], int(sys.argv[3]), sys.argv[4])
+    else:
+        main(sys.argv[1] if len(sys.argv) > 1 else "gpurun_out/ncu_final")
