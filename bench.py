@@ -1103,6 +1103,7 @@ def run_ours(args):
     value = total_bytes / (ms_total * 1e6)
     g = sb.ctx.kernel_stats(aeg.K_GATHER)
     s = sb.ctx.kernel_stats(aeg.K_SCATTER)
+    launches_all = int(dist.sum(g[0] + s[0]))
     hbm, hbm_src = peaks()
     # dominant kernel = gather (HBM bound): algorithmic bytes per launch / mean CUDA-event duration
     g_per_launch_bytes = g[1] / max(1, g[0])
@@ -1122,13 +1123,16 @@ def run_ours(args):
                 sb.step(torch, cons)
                 cons.synchronize()
                 ts.append(time.perf_counter() - t0)
-            e2e_t = statistics.median(ts)
+            e2e_t = dist.max(statistics.median(ts))   # the job's step ends when the slowest rank's does
             e2e = {"value": round(dist.sum(bytes_step) / e2e_t / 1e9, 2), "unit": "GB/s",
                    "h2d_bytes_per_step": int(bytes_step // 2 + 2 * sb.n * 8),
                    "d2h_bytes_per_step": int(bytes_step // 2),
                    "how": "wall clock around the Python-API calls of one step incl. host sync"}
         one_dir = sb.one_direction(torch, cons)
         ver = sb.replay_and_verify()
+        if world > 1:   # every rank checks its own pools; the line reports all of them
+            ver["ranks_failed"] = int(dist.sum(0 if ver["ok"] else 1))
+            ver["ok"] = ver["ranks_failed"] == 0
         sb.ctx.shutdown()
         if args.no_migrate:
             mig = None
@@ -1183,7 +1187,7 @@ def run_ours(args):
                      "peak_per_direction_nominal": PCIE_NOMINAL,
                      "frac_of_duplex_nominal": round(bytes_step / (ms_step * 1e6) / (2 * PCIE_NOMINAL), 3)},
             "clocks": clocks,
-            "gpu_launches": int(g[0] + s[0]),
+            "gpu_launches": launches_all,
             "consumer_launches": args.steps * sb.sh.L,
         }
         res.update(out)
