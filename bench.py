@@ -60,6 +60,9 @@ def parse():
     p.add_argument("--no-switch", action="store_true")
     p.add_argument("--no-migrate", action="store_true")
     p.add_argument("--no-c5", action="store_true", help="skip the configs[4] Qwen-72B TP=4 scale-up leg")
+    # exercise knobs (several ranks sharing one GPU): not used for reported numbers
+    p.add_argument("--c5-model", default="qwen-72b", help=argparse.SUPPRESS)
+    p.add_argument("--churn-slabs", type=int, default=12, help=argparse.SUPPRESS)
     p.add_argument("--no-e2e", action="store_true")
     p.add_argument("--no-cpu", action="store_true")
     p.add_argument("--switches", type=int, default=30)
@@ -208,7 +211,8 @@ def c2_requests(n_req: int):
 class SwapBench:
     """configs[1] on one GPU: aged device pool, a 64-request batch, swap round trips."""
 
-    def __init__(self, aeg, sh, n_req, kernel, extra_host_slabs=8, weight_bytes=0, seed_cfg=2, slot_mib=0, slots=0):
+    def __init__(self, aeg, sh, n_req, kernel, extra_host_slabs=8, weight_bytes=0, seed_cfg=2, slot_mib=0, slots=0,
+                 churn_slabs=12):
         import aeg_inputs as gi
         from oracle import kv as OK
         from oracle.shape import KVShape
@@ -222,7 +226,7 @@ class SwapBench:
         self.n = len(self.labels)
         self.k = GIB // self.sh.block_bytes()
         batch_slabs = -(-self.n // self.k)
-        self.churn_slabs = 12
+        self.churn_slabs = churn_slabs
         dev_slabs = 2 * batch_slabs + self.churn_slabs + 4
         host_slabs = batch_slabs + extra_host_slabs
         self.seed = gi.kv_seed(seed_cfg)
@@ -811,7 +815,7 @@ def _c5_check_weights(aeg, ctx, name, m, seed, tp_rank, tp_size, got_offs, picks
     return ok and bad == 0, len(picks)
 
 
-def c5_leg(aeg, torch, kernel, dist=None, tp_rank=1, tp_size=4, reps=3):
+def c5_leg(aeg, torch, kernel, dist=None, tp_rank=1, tp_size=4, reps=3, model="qwen-72b"):
     """configs[4]: Qwen-72B TP=4 scale-up.  The decode instance's rank r stages its 36.1 GB weight
     shard (Megatron col/row/vocab split, host threads -> pinned Stage Buffer -> PCIe, PAPER.md:
     1343-1354) while its prefill partner hands it 2 GiB of KV (Qwen-72B-TP4 shape, H=16 per rank)
@@ -836,13 +840,13 @@ def c5_leg(aeg, torch, kernel, dist=None, tp_rank=1, tp_size=4, reps=3):
     n_kv = (2 * GIB) // sh.block_bytes()
     slab = 10 * 64 * MIB * 2            # 1.25 GiB: 128 blocks of 10 MiB
     nslab = -(-n_kv // (slab // sh.block_bytes())) + 1
-    out = {"workload": "configs[4] Qwen-72B TP=4 scale-up: one decode rank stages its weight shard (staged 3.a) "
+    out = {"workload": f"configs[4] {model} TP=4 scale-up: one decode rank stages its weight shard (staged 3.a) "
                        f"while its prefill partner migrates {n_kv} blocks ({n_kv * sh.block_bytes() / GIB:.2f} GiB) "
                        "of KV to it" + (" (1 GPU: both ranks' contexts on it)" if world == 1 else f", {world} ranks")}
     descs, keep, touched, wctx, a, b = None, None, 0, None, None, None
     t0 = time.time()
     if decode:
-        descs, keep, touched = sparse_model_cache("qwen-72b", 7, tp_rank, tp_size, seed_w)
+        descs, keep, touched = sparse_model_cache(model, 7, tp_rank, tp_size, seed_w)
         shard_total = sum(-(-(d["rows"] * d["cols"] * 2 // (1 if d["split"] == gi.REPLICATED else tp_size)) // 256) * 256
                           for d in descs)
         wctx = aeg.Context(device, aeg.default_config(device_kv_bytes=nslab * slab, host_kv_bytes=GIB,
@@ -918,7 +922,7 @@ def c5_leg(aeg, torch, kernel, dist=None, tp_rank=1, tp_size=4, reps=3):
         offs, x = b.weights_stage(descs, tp_rank, tp_size)
         b.layer_ready(x, -1, aeg.READY_BLOCK)
         b.xfer_release(x)
-        w_ok, picks = _c5_check_weights(aeg, b, "qwen-72b", 7, seed_w, tp_rank, tp_size, offs, pick)
+        w_ok, picks = _c5_check_weights(aeg, b, model, 7, seed_w, tp_rank, tp_size, offs, pick)
     kv_bad = 0
     if decode:
         sender = 0 if world == 1 else rank - world // 2
@@ -938,6 +942,9 @@ def c5_leg(aeg, torch, kernel, dist=None, tp_rank=1, tp_size=4, reps=3):
         shard = dist.max(shard)
         kv_bad = dist.sum(kv_bad)
         w_ok = dist.sum(0 if w_ok else 1) == 0
+        picks = int(dist.sum(picks))
+        out["model_cache_build_s"] = round(dist.max(out["model_cache_build_s"]), 1)
+        out["model_cache_touched_bytes"] = int(dist.max(touched))
     kvb = n_kv * sh.block_bytes()
     wm, km, bm = statistics.median(w_ms), statistics.median(k_ms), statistics.median(both)
     out.update({"tp_size": tp_size, "decode_ranks": n_dec, "shard_bytes_per_rank": int(shard),
@@ -1079,7 +1086,8 @@ def run_ours(args):
         per_rank = psutil.virtual_memory().available / world
         while n_req > 4 and sum(c2_requests(n_req)[1]) * 8 * MIB * 1.3 > per_rank:
             n_req //= 2
-    sb = SwapBench(aeg, QWEN7B, n_req, kernel, slot_mib=args.slot_mib, slots=args.slots).setup()
+    sb = SwapBench(aeg, QWEN7B, n_req, kernel, slot_mib=args.slot_mib, slots=args.slots,
+                   churn_slabs=args.churn_slabs).setup()
     sb.sink = torch.zeros(1, dtype=torch.int64, device="cuda")
     cons = torch.cuda.Stream()
     bytes_step = 2 * sb.n * sb.sh.block_bytes()
@@ -1154,7 +1162,7 @@ def run_ours(args):
         if args.no_c5:
             c5 = None
         elif world in (1, 8):
-            c5 = c5_leg(aeg, torch, kernel, dist if world > 1 else None)
+            c5 = c5_leg(aeg, torch, kernel, dist if world > 1 else None, model=args.c5_model)
         else:
             c5 = {"skipped": "configs[4] is the 8-GPU TP=4 layout (one rank pair on 1 GPU); not defined for N=%d" % world}
         cpu = None if args.no_cpu or rank != 0 else cpu_baseline()
