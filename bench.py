@@ -959,6 +959,58 @@ def c5_leg(aeg, torch, kernel, dist=None, tp_rank=1, tp_size=4, reps=3, model="q
     return out
 
 
+def allocator_leg(aeg, reps=20):
+    """H1 control overhead ("tracking indices in the unified cache"): the slab
+    allocator of a host-only context with the C2 geometry (82 GiB device pool, 1 GiB slabs, aged by
+    the same churn), timed per aeg_kv_alloc / aeg_kv_free call through the Python binding (the
+    1-block call shows the binding's own per-call cost)."""
+    import aeg_inputs as gi
+    cfg = aeg.default_config(device_kv_bytes=82 * GIB, host_kv_bytes=40 * GIB,
+                             flags=aeg.CFG_HOST_ONLY | aeg.CFG_NO_DAEMON)
+    ctx = aeg.Context(0, cfg)
+    sh = QWEN7B
+    _, blocks = c2_requests(64)
+    live = []
+    for op, v in gi.churn_ops(2, capacity_blocks=12 * (GIB // (8 * MIB)), hi_blocks=96):
+        if op == "alloc":
+            live.append(ctx.kv_alloc(0, sh, v))
+        elif live[v] is not None:
+            ctx.kv_free(0, live[v])
+            live[v] = None
+    pa, pf, ba, bf, one = [], [], [], [], []
+    clk = time.perf_counter_ns
+    for _ in range(reps):
+        hs = []
+        for b in blocks:
+            t0 = clk()
+            hs.append(ctx.kv_alloc(0, sh, b))
+            pa.append(clk() - t0)
+        for h in hs:
+            t0 = clk()
+            ctx.kv_free(0, h)
+            pf.append(clk() - t0)
+        t0 = clk()
+        h = ctx.kv_alloc(0, sh, sum(blocks))
+        t1 = clk()
+        ctx.kv_free(0, h)
+        ba.append(t1 - t0)
+        bf.append(clk() - t1)
+    for _ in range(1000):
+        t0 = clk()
+        h = ctx.kv_alloc(0, sh, 1)
+        one.append(clk() - t0)
+        ctx.kv_free(0, h)
+    ctx.shutdown()
+    n = sum(blocks)
+    med = lambda v: round(statistics.median(v) / 1e3, 2)  # noqa: E731
+    return {"workload": f"C2 geometry, aged pool; 64 per-request calls ({n} Qwen-7B blocks) and one {n}-block call",
+            "per_request_alloc_us_p50": med(pa), "per_request_free_us_p50": med(pf),
+            "batch_alloc_us": med(ba), "batch_free_us": med(bf),
+            "batch_alloc_ns_per_block": round(statistics.median(ba) / n, 1),
+            "batch_free_ns_per_block": round(statistics.median(bf) / n, 1),
+            "one_block_call_us_p50": med(one), "includes": "Python ctypes call overhead"}
+
+
 def overlap_leg(aeg, torch, kernel, work_us=500, reps=5):
     """North star: "decoding of layer i overlaps the transfer of layer i+1".  A 1 GiB Llama-7B KV
     batch (32 layers) is swapped in while a synthetic decode step does `work_us` of work per layer
@@ -1165,9 +1217,10 @@ def run_ours(args):
             c5 = c5_leg(aeg, torch, kernel, dist if world > 1 else None, model=args.c5_model)
         else:
             c5 = {"skipped": "configs[4] is the 8-GPU TP=4 layout (one rank pair on 1 GPU); not defined for N=%d" % world}
+        alloc = allocator_leg(aeg) if rank == 0 else None
         cpu = None if args.no_cpu or rank != 0 else cpu_baseline()
         out.update({"e2e": e2e, "verify": ver, "one_direction": one_dir, "pcie_memcpy_GBps": {k: round(v, 1) for k, v in pc.items()},
-                    "switch": sw, "migrate": mig, "per_layer_overlap": ovl, "c5": c5,
+                    "switch": sw, "migrate": mig, "per_layer_overlap": ovl, "c5": c5, "allocator": alloc,
                     "cpu_baseline": cpu})
         if not ver["ok"]:
             log("VERIFICATION FAILED", ver)
