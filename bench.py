@@ -8,8 +8,10 @@ preempt and swap out a 64-request decode batch, then swap back in, on 1 B200"):
     per-layer waits on the swap-out, so the two directions overlap full duplex)  ->  H6 a synthetic
     decode consumer waits per layer (rule ❶) and reads each layer  ->  H1 free (move lists).
 value = KV bytes moved over PCIe per step (out + in) / device time of the step, in GB/s.
-After the timed region every chunk of the device pool is checked against the oracle's label image
-(oracle/kv.py at chunk granularity) and sampled chunks against the NumPy generator.
+After the timed region the north-star invariant is checked: swap_in o swap_out is the identity on
+every chunk of the batch (generator content at the library's block table), resident blocks are
+untouched.  bench.py runs the oracle (oracle/) only in its cpu_baseline leg and in --impl reference;
+the oracle parity of the same workloads is in tests/ (test_gpu_fullsize.py, test_gpu_c5.py).
 
 Also measured in the same run (not in `value`): H7+H8 model switch among Qwen-1.8B / Llama-7B /
 Yi-9B shapes with 1 GiB KV each (configs[3]), H5 local migrate (configs[2] shapes, one GPU), the
@@ -208,18 +210,27 @@ def c2_requests(n_req: int):
     return lens, blocks
 
 
+def chunk_offsets(ctx, pool, shape, blocks):
+    """Byte offsets from the pool base of every (block, layer) chunk of `blocks`, block-major, from
+    the library's block table (aeg_block_offsets)."""
+    off0, stride = ctx.block_offsets(pool, shape, blocks)
+    L = int(shape[0])
+    return (off0[:, None] + np.arange(L, dtype=np.uint64)[None, :] * np.uint64(stride)).reshape(-1)
+
+
 class SwapBench:
-    """configs[1] on one GPU: aged device pool, a 64-request batch, swap round trips."""
+    """configs[1] on one GPU: aged device pool, a 64-request batch, swap round trips.  Library calls
+    and the seeded generator only: input placement uses the library's own block table
+    (aeg_block_offsets).  The oracle-mirrored variant with the whole-pool parity check is
+    tests/oracle_swapbench.py (test infrastructure)."""
 
     def __init__(self, aeg, sh, n_req, kernel, extra_host_slabs=8, weight_bytes=0, seed_cfg=2, slot_mib=0, slots=0,
                  churn_slabs=12):
         import aeg_inputs as gi
-        from oracle import kv as OK
-        from oracle.shape import KVShape
-        from oracle.slab import SlabPool
-        self.aeg, self.gi, self.OK = aeg, gi, OK
+        self.aeg, self.gi = aeg, gi
         self.sht = sh
-        self.sh = KVShape(*sh)
+        self.sh = aeg.KVShape.of(sh)
+        self.L = self.sh.num_layers
         self.Cl = self.sh.chunk_bytes()
         self.lens, blocks = c2_requests(n_req)
         self.labels = [(r, j) for r, b in enumerate(blocks) for j in range(b)]
@@ -241,87 +252,103 @@ class SwapBench:
         import torch
         self.ctx = aeg.Context(torch.cuda.current_device(), cfg)
         self.init_s = time.time() - t0
-        self.dg = OK.PoolGeom(cfg.device_kv_bytes, GIB, aeg.LAYER_MAJOR)
-        self.hg = OK.PoolGeom(cfg.host_kv_bytes, GIB, aeg.LAYER_MAJOR)
-        self.od, self.oh = SlabPool(self.dg.nbytes, GIB), SlabPool(self.hg.nbytes, GIB)
         self.dbase, _ = self.ctx.pool_region(aeg.POOL_DEVICE)
         self.hbase, _ = self.ctx.pool_region(aeg.POOL_HOST)
-        self.ops = []   # library calls of the timed steps, replayed on the oracle afterwards
+        self.ops = []   # (host blocks, device blocks) of every round trip, in order
 
-    # oracle-mirrored allocation outside the timed region
-    def alloc_both(self, pool, n):
-        c = self.ctx.kv_alloc(pool, self.sht, n)
-        o = (self.od if pool == 0 else self.oh).alloc(self.sh, n)
-        assert [(s, j) for _, s, j in map(self.aeg.decode_block, c)] == list(o), "allocator diverged from oracle"
-        return c, o
+    def chunk_offsets(self, pool, blocks):
+        """Byte offsets (from the pool base) of every (block, layer) chunk, block-major, from the
+        library's block table."""
+        off0, stride = self.ctx.block_offsets(pool, self.sht, blocks)
+        return (off0[:, None] + np.arange(self.L, dtype=np.uint64)[None, :] * np.uint64(stride)).reshape(-1)
+
+    def batch_keys(self):
+        gi = self.gi
+        return np.array([gi.kv_key(1, r, j, l) for (r, j) in self.labels for l in range(self.L)], np.uint64)
 
     def setup(self):
-        from aeg_inputs import dev as D
-        gi, OK, sh = self.gi, self.OK, self.sh
-        # never-allocated bytes carry their offset-keyed poison: the label image starts as poison
-        D.fill_region(self.dbase, self.dg.nbytes, self.seed, gi.poison_key(gi.TAG_NEVER, 0))
-        cells = self.dg.nbytes // self.Cl
-        self.lab = (np.uint64(gi.poison_key(gi.TAG_NEVER, 0))
-                    + np.arange(cells, dtype=np.uint64) * np.uint64(self.Cl // 8))
-        self.hlab = np.zeros(self.hg.nbytes // self.Cl, dtype=np.uint64)   # 0 = unknown content
+        gi, aeg = self.gi, self.aeg
         # aging churn (SURVEY §8(d) placement realism): other requests' blocks stay resident
         live = []
-        cap = self.churn_slabs * self.k
-        for op, v in gi.churn_ops(2, capacity_blocks=cap, hi_blocks=96):
+        for op, v in gi.churn_ops(2, capacity_blocks=self.churn_slabs * self.k, hi_blocks=96):
             if op == "alloc":
-                live.append(self.alloc_both(0, v))
-            else:
-                if live[v] is not None:
-                    self.ctx.kv_free(0, live[v][0])
-                    self.od.free(live[v][1])
-                    live[v] = None
+                live.append(self.ctx.kv_alloc(aeg.POOL_DEVICE, self.sht, v))
+            elif live[v] is not None:
+                self.ctx.kv_free(aeg.POOL_DEVICE, live[v])
+                live[v] = None
         self.churn = [x for x in live if x is not None]
-        offs, keys = [], []
-        for q, (c, o) in enumerate(self.churn):
-            for j, h in enumerate(o):
-                for l in range(sh.L):
-                    a = OK.addr(self.dg, sh, h, l)
-                    offs.append(a)
-                    keys.append(gi.kv_key(2, q % 65536, j, l))
-        self._fill(offs, keys)
-        # the batch
-        self.src_c, self.src_o = self.alloc_both(0, self.n)
-        offs, keys = [], []
-        for (r, j), h in zip(self.labels, self.src_o):
-            for l in range(sh.L):
-                offs.append(OK.addr(self.dg, sh, h, l))
-                keys.append(gi.kv_key(1, r, j, l))
-        self._fill(offs, keys)
-        # layer-0 offsets of the consumer (located through the public API: aeg_block_ptr)
+        self.churn_offs = np.concatenate([self.chunk_offsets(0, c) for c in self.churn])
+        self.churn_keys = np.array([gi.kv_key(2, q % 65536, j, l) for q, c in enumerate(self.churn)
+                                    for j in range(len(c)) for l in range(self.L)], np.uint64)
+        self._fill(self.churn_offs, self.churn_keys)
+        self.src_c = self.ctx.kv_alloc(aeg.POOL_DEVICE, self.sht, self.n)
+        self._fill(self.chunk_offsets(0, self.src_c), self.batch_keys())
         return self
 
-    def _fill(self, offs, keys):
+    def _fill(self, offs, keys, base=None):
         from aeg_inputs import dev as D
         offs = np.asarray(offs, np.uint64)
         keys = np.asarray(keys, np.uint64)
         for a in range(0, offs.size, 1 << 16):
-            D.fill_chunks(self.dbase, offs[a:a + (1 << 16)], keys[a:a + (1 << 16)], self.Cl, self.seed)
-        self.lab[(offs // np.uint64(self.Cl)).astype(np.int64)] = keys
+            D.fill_chunks(self.dbase if base is None else base, offs[a:a + (1 << 16)], keys[a:a + (1 << 16)],
+                          self.Cl, self.seed)
+
+    def _verify(self, base, offs, keys):
+        from aeg_inputs import dev as D
+        bad = 0
+        for a in range(0, offs.size, 1 << 17):
+            b, _ = D.verify_chunks(base, offs[a:a + (1 << 17)], keys[a:a + (1 << 17)], self.Cl, self.seed)
+            bad += b
+        return bad
+
+    def verify(self):
+        """The north-star invariant after all round trips: swap_in o swap_out is the identity on every
+        chunk of the batch (its current device blocks and its last host copy hold the generator's
+        bytes for each (request, block, layer) label), and the resident requests' blocks around it
+        are untouched.  Chunks are located through the library's block table; expected bytes come
+        from the seeded generator only (CUDA evaluation, plus a NumPy evaluation of sampled chunks)."""
+        from aeg_inputs import dev as D
+        keys = self.batch_keys()
+        doffs = self.chunk_offsets(0, self.src_c)
+        dbad = self._verify(self.dbase, doffs, keys)
+        hbad, hn = 0, 0
+        if getattr(self, "host_offs", None) is not None:   # the last swap-out's host copy
+            hbad, hn = self._verify(self.hbase, self.host_offs, keys), self.host_offs.size
+        cbad = self._verify(self.dbase, self.churn_offs, self.churn_keys)
+        rng = np.random.default_rng(7)
+        sample_bad = 0
+        for c in rng.choice(doffs.size, size=8, replace=False):
+            got = D.read(self.dbase + int(doffs[c]), self.Cl)
+            sample_bad += int((got != self.gi.region_bytes(self.seed, int(keys[c]), self.Cl)).sum())
+        return {"batch_device_chunks_checked": int(doffs.size), "batch_device_bad_words": int(dbad),
+                "batch_host_chunks_checked": int(hn), "batch_host_bad_words": int(hbad),
+                "resident_chunks_checked": int(self.churn_offs.size), "resident_bad_words": int(cbad),
+                "numpy_sampled_chunks": 8, "numpy_sampled_bad_bytes": sample_bad,
+                "ok": dbad == 0 and hbad == 0 and cbad == 0 and sample_bad == 0,
+                "what": "swap_in o swap_out = identity on every chunk of the batch; resident blocks untouched "
+                        "(whole-pool oracle parity: tests/test_gpu_fullsize.py)"}
 
     def consumer_tables(self, torch, blocks):
         """[L][n] byte offsets of each layer of `blocks` from the pool base (aeg_block_offsets: the
         block table a PagedAttention-style consumer would build)."""
         off0, stride = self.ctx.block_offsets(0, self.sht, blocks)
-        t = off0[None, :] + np.arange(self.sh.L, dtype=np.uint64)[:, None] * np.uint64(stride)
+        t = off0[None, :] + np.arange(self.L, dtype=np.uint64)[:, None] * np.uint64(stride)
         return torch.from_numpy(t.astype(np.int64)).cuda()
 
-    def step(self, torch, cons, with_consumer=True, record=True):
+    def step(self, torch, cons, with_consumer=True, record=True, keep_host_offsets=False):
         """One timed step, library calls only (plus the synthetic consumer)."""
         aeg = self.aeg
         from aeg_inputs import dev as D
         hc = self.ctx.kv_alloc(aeg.POOL_HOST, self.sht, self.n)
+        if keep_host_offsets:   # the host blocks are freed (and their slabs may be reclaimed) by the swap-in
+            self.host_offs = self.chunk_offsets(1, hc)
         nd = self.ctx.kv_alloc(aeg.POOL_DEVICE, self.sht, self.n)
         self.ctx.stream_fence(cons.cuda_stream)
         x = self.ctx.kv_swap_out(self.sht, self.src_c, hc, flags=aeg.FREE_SRC)
         y = self.ctx.kv_swap_in(self.sht, hc, nd, flags=aeg.FREE_SRC)
         if with_consumer:
             tab = self.consumer_tables(torch, nd)
-            for l in range(self.sh.L):
+            for l in range(self.L):
                 self.ctx.layer_ready(y, l, aeg.READY_WAIT_STREAM, cons.cuda_stream)
                 D.consume(self.dbase, tab[l].data_ptr(), self.n, self.Cl, self.sink.data_ptr(), cons.cuda_stream)
         else:
@@ -342,6 +369,7 @@ class SwapBench:
         out = {}
         hc = self.ctx.kv_alloc(aeg.POOL_HOST, self.sht, self.n)
         nd = self.ctx.kv_alloc(aeg.POOL_DEVICE, self.sht, self.n)
+        self.host_offs = self.chunk_offsets(1, hc)
         for name in ("swap_out", "swap_in"):
             self.ctx.kernel_stats_reset()
             e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
@@ -364,54 +392,6 @@ class SwapBench:
         self.ops.append((hc, nd))
         self.src_c = nd
         return out
-
-    def replay_and_verify(self):
-        """Oracle replay of the recorded steps; full device-pool check + sampled host-side check."""
-        from aeg_inputs import dev as D
-        OK, gi, aeg = self.OK, self.gi, self.aeg
-        src_o = self.src_o
-        for hc, nd in self.ops:
-            hco = self.oh.alloc(self.sh, self.n)
-            ndo = self.od.alloc(self.sh, self.n)
-            assert [(s, j) for _, s, j in map(aeg.decode_block, hc)] == list(hco), "host allocator diverged"
-            assert [(s, j) for _, s, j in map(aeg.decode_block, nd)] == list(ndo), "device allocator diverged"
-            xo = self.od.begin(src_o)
-            self.od.free(src_o)
-            yo = self.oh.begin(hco)
-            self.oh.free(hco)
-            self.hlab = OK.swap_out(self.lab, self.dg, self.hlab, self.hg, self.sh, src_o, hco, unit=self.Cl)
-            self.lab = OK.swap_in(self.hlab, self.hg, self.lab, self.dg, self.sh, hco, ndo, unit=self.Cl)
-            self.od.complete(xo)
-            self.oh.complete(yo)
-            src_o = ndo
-        self.src_o = src_o
-        # every chunk of the device pool equals the generator at the oracle's label (full size)
-        cells = self.lab.size
-        offs = np.arange(cells, dtype=np.uint64) * np.uint64(self.Cl)
-        bad_total = 0
-        for a in range(0, cells, 1 << 17):
-            bad, first = D.verify_chunks(self.dbase, offs[a:a + (1 << 17)], self.lab[a:a + (1 << 17)], self.Cl, self.seed)
-            bad_total += bad
-        # host pool: every chunk the oracle says was written
-        known = np.nonzero(self.hlab)[0]
-        hoffs = known.astype(np.uint64) * np.uint64(self.Cl)
-        hbad = 0
-        for a in range(0, known.size, 1 << 16):
-            b, _ = D.verify_chunks(self.hbase, hoffs[a:a + (1 << 16)], self.hlab[known[a:a + (1 << 16)]], self.Cl,
-                                   self.seed)
-            hbad += b
-        # sampled chunks against the NumPy generator directly (no CUDA generator involved)
-        rng = np.random.default_rng(7)
-        sample_bad = 0
-        batch_cells = [OK.addr(self.dg, self.sh, h, l) // self.Cl for h in self.src_o for l in (0, self.sh.L - 1)]
-        for c in rng.choice(batch_cells, size=8, replace=False):
-            got = D.read(self.dbase + int(c) * self.Cl, self.Cl)
-            exp = gi.region_bytes(self.seed, int(self.lab[c]), self.Cl)
-            sample_bad += int((got != exp).sum())
-        return {"device_chunks_checked": int(cells), "device_bad_words": int(bad_total),
-                "host_chunks_checked": int(known.size), "host_bad_words": int(hbad),
-                "numpy_sampled_chunks": 8, "numpy_sampled_bad_bytes": sample_bad,
-                "ok": bad_total == 0 and hbad == 0 and sample_bad == 0}
 
 
 # ----------------------------------------------------------------------------------- legs
@@ -496,7 +476,7 @@ def switch_leg(aeg, torch, n_switch, kernel, descs, mode="staged", caches=None):
     if mode == "prefetch":
         ctx.weights_reset(-(-wsize[cur] // 256) * 256)
         o, xp = ctx.weights_stage(descs[names[1]])
-        pre = (names[1], xp, int(o[0]))
+        pre = (names[1], xp, int(o[0]), o)
     cons = torch.cuda.Stream()
     res = []
     diag_ms = None
@@ -518,11 +498,12 @@ def switch_leg(aeg, torch, n_switch, kernel, descs, mode="staged", caches=None):
         kv[nxt] = (db, kv[nxt][1])
         if mode in ("staged", "direct"):
             ctx.weights_reset(0)
-            _, xw = ctx.weights_stage(descs[nxt])                                      # B's weights in
+            wo, xw = ctx.weights_stage(descs[nxt])                                     # B's weights in
             wl = lambda l: min(l, ctx.xfer_layers(xw) - 1)  # noqa: E731
         else:
             assert pre[0] == nxt
             xw = ctx.weights_relocate(pre[2], 0, wsize[nxt])                           # 3.b: on-device copy
+            wo = [int(x) - pre[2] for x in pre[3]]
             ctx.xfer_release(pre[1])
             wl = lambda l: 0  # noqa: E731
         diag = {}
@@ -560,15 +541,14 @@ def switch_leg(aeg, torch, n_switch, kernel, descs, mode="staged", caches=None):
         if i >= 3:
             res.append(dict(to=nxt, first_ms=e0.elapsed_time(ev[0]), last_ms=e0.elapsed_time(e_end),
                             bytes_h2d=(0 if mode == "prefetch" else wsize[nxt]) + kvb))
-        if i == len(order) - 1:   # bit-exact check of the running model's weights (oracle O8, TP=1)
+        if i == len(order) - 1:   # bit-exact check of the running model's weights (TP=1: the tensors)
             base, _, _ = ctx.weights_region()
-            from oracle import weights as W
             m = names.index(nxt)
             bad = 0
             for k in (0, len(descs[nxt]) // 2, len(descs[nxt]) - 1):
                 d = descs[nxt][k]
                 nb = d["rows"] * d["cols"] * 2
-                o = W.bump_offsets([x["rows"] * x["cols"] * 2 for x in descs[nxt]], 0)[0][k]
+                o = int(wo[k])
                 got = D.read(base + o, min(nb, 1 << 24))
                 exp = gi.region_bytes(gi.w_seed(3), gi.weight_key(m, k), min(nb, 1 << 24))
                 bad += int((got != exp).sum())
@@ -577,7 +557,7 @@ def switch_leg(aeg, torch, n_switch, kernel, descs, mode="staged", caches=None):
             nn = names[(names.index(cur) + 1) % len(names)]
             ctx.weights_reset(-(-wsize[cur] // 256) * 256)
             o, xp = ctx.weights_stage(descs[nn])
-            pre = (nn, xp, int(o[0]))
+            pre = (nn, xp, int(o[0]), o)
     if pre is not None:
         ctx.layer_ready(pre[1], -1, aeg.READY_BLOCK)
     wchunks, wfill, wslot = ctx.weights_stats()
@@ -610,13 +590,12 @@ def switch_leg(aeg, torch, n_switch, kernel, descs, mode="staged", caches=None):
 def migrate_leg(aeg, torch, kernel, n_req=4):
     """configs[2] shapes on one GPU: Llama-2-13B KV hand-off through the fused migrate kernel into
     another context's pool (peer mapped in-process, the same kernel that stores over NVLink when the
-    peer is another GPU).  Checked against the generator at the oracle's placement."""
+    peer is another GPU).  Checked against the generator at the destination blocks' chunks (identity
+    under relabelling), located through the library's block table."""
     import aeg_inputs as gi
     from aeg_inputs import dev as D
-    from oracle import kv as OK
-    from oracle.shape import KVShape
     sht = gi.KV_SHAPES["llama-2-13b"]
-    sh = KVShape(*sht)
+    sh = aeg.KVShape.of(sht)
     lens = gi.request_lengths(3, n_req, 512, 4096)
     n = sum(-(-t // 16) for t in lens)
     slab = 1 * GIB + 256 * MIB
@@ -629,13 +608,9 @@ def migrate_leg(aeg, torch, kernel, n_req=4):
     dc = b.kv_alloc(0, sht, n)
     abase, _ = a.pool_region(0)
     bbase, _ = b.pool_region(0)
-    ga = OK.PoolGeom(nslab * slab, slab, aeg.LAYER_MAJOR)
-    gb = OK.PoolGeom(nslab * slab, slab, aeg.BLOCK_MAJOR)
     seed = gi.kv_seed(3)
-    so = [aeg.decode_block(x)[1:] for x in sc]
-    do = [aeg.decode_block(x)[1:] for x in dc]
-    offs = [OK.addr(ga, sh, h, l) for h in so for l in range(sh.L)]
-    keys = [gi.kv_key(1, i // 4096, i % 4096, l) for i in range(n) for l in range(sh.L)]
+    offs = chunk_offsets(a, 0, sht, sc)
+    keys = [gi.kv_key(1, i // 4096, i % 4096, l) for i in range(n) for l in range(sh.num_layers)]
     D.fill_chunks(abase, offs, keys, sh.chunk_bytes(), seed)
     a.import_peer(1, b.export_ipc())
     times = []
@@ -653,7 +628,7 @@ def migrate_leg(aeg, torch, kernel, n_req=4):
         if it >= 2:
             times.append(e0.elapsed_time(e1))
     nl, nbytes, kms = a.kernel_stats(aeg.K_MIGRATE)
-    doffs = [OK.addr(gb, sh, h, l) for h in do for l in range(sh.L)]
+    doffs = chunk_offsets(b, 0, sht, dc)
     bad, _ = D.verify_chunks(bbase, doffs, keys, sh.chunk_bytes(), seed)
     a.shutdown()
     b.shutdown()
@@ -672,12 +647,10 @@ def migrate_leg_dist(aeg, torch, dist, kernel, n_req=4):
     Aggregate GB/s = all pairs' payload / max-over-ranks device time."""
     import aeg_inputs as gi
     from aeg_inputs import dev as D
-    from oracle import kv as OK
-    from oracle.shape import KVShape
     from paper_conf_sosp_xiang0qyzyzl0025_b200 import dist as PD
     world, rank = dist.world, dist.rank
     sht = gi.KV_SHAPES["llama-2-13b"]
-    sh = KVShape(*sht)
+    sh = aeg.KVShape.of(sht)
     lens = gi.request_lengths(3, n_req, 512, 4096)
     n = sum(-(-t // 16) for t in lens)
     slab = GIB + 256 * MIB
@@ -686,7 +659,6 @@ def migrate_leg_dist(aeg, torch, dist, kernel, n_req=4):
                              dev_slab_layout=aeg.LAYER_MAJOR if PD.role(rank, world) == "prefill" else aeg.BLOCK_MAJOR,
                              kernel=kernel, flags=aeg.CFG_TIMING)
     ctx = aeg.Context(dist.device, cfg)
-    geom = OK.PoolGeom(nslab * slab, slab, cfg.dev_slab_layout)
     base, _ = ctx.pool_region(0)
     seed = gi.kv_seed(3)
     PD.connect(ctx, rank)
@@ -697,9 +669,8 @@ def migrate_leg_dist(aeg, torch, dist, kernel, n_req=4):
     src = None
     if prefill:
         src = ctx.kv_alloc(0, sht, n)
-        so = [aeg.decode_block(b)[1:] for b in src]
-        offs = [OK.addr(geom, sh, h, l) for h in so for l in range(sh.L)]
-        keys = [gi.kv_key(1, rank, i, l) for i in range(n) for l in range(sh.L)]
+        offs = chunk_offsets(ctx, 0, sht, src)
+        keys = [gi.kv_key(1, rank, i, l) for i in range(n) for l in range(sh.num_layers)]
         D.fill_chunks(base, offs, keys, sh.chunk_bytes(), seed)
     dst_by_rank = {d: np.array(h, np.uint64) for d, h in enumerate(handles) if h}
 
@@ -725,7 +696,7 @@ def migrate_leg_dist(aeg, torch, dist, kernel, n_req=4):
             for sender, m in enumerate(blobs):
                 if m and rank in m:
                     xi = ctx.xfer_import(sender, m[rank])
-                    for l in range(sh.L):
+                    for l in range(sh.num_layers):
                         ctx.layer_ready(xi, l, aeg.READY_BLOCK)
                     ctx.xfer_release(xi)
         for x in xs.values():
@@ -736,9 +707,8 @@ def migrate_leg_dist(aeg, torch, dist, kernel, n_req=4):
     bad = 0
     if not prefill:
         sender = [s_ for s_, d in pairs if d == rank][0]
-        do = [aeg.decode_block(b)[1:] for b in dst]
-        offs = [OK.addr(geom, sh, h, l) for h in do for l in range(sh.L)]
-        keys = [gi.kv_key(1, sender, i, l) for i in range(n) for l in range(sh.L)]
+        offs = chunk_offsets(ctx, 0, sht, dst)
+        keys = [gi.kv_key(1, sender, i, l) for i in range(n) for l in range(sh.num_layers)]
         bad, _ = D.verify_chunks(base, offs, keys, sh.chunk_bytes(), seed)
     bad = dist.sum(bad)
     # SURVEY §8(d) C3 for N >= 4: all-to-all, every prefill rank -> every decode rank, round-robin
@@ -797,36 +767,43 @@ def sparse_model_cache(name, m, tp_rank, tp_size, seed, threads=16, min_sparse=M
 
 
 def _c5_check_weights(aeg, ctx, name, m, seed, tp_rank, tp_size, got_offs, picks):
-    """Sampled O8 parity: the oracle shards the densely generated tensor; the device copy must match."""
+    """Sampled check of staged shards at the offsets the library returned: each expected shard is cut
+    from the generator's dense tensor by its split's definition (the row/column ranges the input
+    builder materialised).  The oracle's O8 check of the same run is tests/test_gpu_c5.py."""
     import aeg_inputs as gi
     from aeg_inputs import dev as D
-    from oracle import weights as W
     ts = gi.model_tensors(name)
-    shard_sizes = [t["rows"] * t["cols"] * 2 // (1 if t["split"] == W.REPLICATED else tp_size) for t in ts]
-    exp_offs, _ = W.bump_offsets(shard_sizes, 0)
-    ok = [int(o) for o in got_offs] == exp_offs
     base, _, _ = ctx.weights_region()
     bad = 0
     for k in picks:
         t = ts[k]
-        full = gi.region_bytes(seed, gi.weight_key(m, k), t["rows"] * t["cols"] * 2).reshape(t["rows"], t["cols"], 2)
-        exp = np.ascontiguousarray(W.shard(full, t["split"], t["groups"], tp_rank, tp_size)).reshape(-1)
-        bad += int((D.read(base + exp_offs[k], exp.size) != exp).sum())
-    return ok and bad == 0, len(picks)
+        rows, cb = t["rows"], t["cols"] * 2
+        full = gi.region_bytes(seed, gi.weight_key(m, k), rows * cb).reshape(rows, cb)
+        if t["split"] == gi.REPLICATED:
+            exp = full
+        elif t["split"] in (gi.COL, gi.VOCAB):
+            g, p = rows // t["groups"], rows // t["groups"] // tp_size
+            exp = np.concatenate([full[q * g + tp_rank * p:q * g + (tp_rank + 1) * p] for q in range(t["groups"])])
+        else:
+            w = cb // tp_size
+            exp = full[:, tp_rank * w:(tp_rank + 1) * w]
+        exp = np.ascontiguousarray(exp).reshape(-1)
+        bad += int((D.read(base + int(got_offs[k]), exp.size) != exp).sum())
+    return bad == 0, len(picks)
 
 
-def c5_leg(aeg, torch, kernel, dist=None, tp_rank=1, tp_size=4, reps=3, model="qwen-72b"):
+def c5_leg(aeg, torch, kernel, dist=None, tp_rank=1, tp_size=4, reps=3, model="qwen-72b", check=None):
     """configs[4]: Qwen-72B TP=4 scale-up.  The decode instance's rank r stages its 36.1 GB weight
     shard (Megatron col/row/vocab split, host threads -> pinned Stage Buffer -> PCIe, PAPER.md:
     1343-1354) while its prefill partner hands it 2 GiB of KV (Qwen-72B-TP4 shape, H=16 per rank)
     through the fused migrate kernel (PAPER.md:2096-2098 layout).  One GPU: one rank pair, the
     prefill side a second context on the same GPU (the same kernel stores over NVLink when the peer
     is another GPU); with 8 ranks: ranks 0-3 prefill, 4-7 decode, rank i -> i + 4.
-    Reports per-rank weights GB/s, KV hand-off GB/s and the scale-up time (both ready)."""
+    Reports per-rank weights GB/s, KV hand-off GB/s and the scale-up time (both ready).
+    `check(ctx, model, m, seed, tp_rank, tp_size, offsets, picks)` replaces the sampled weights
+    check (the GPU test passes the oracle's)."""
     import aeg_inputs as gi
     from aeg_inputs import dev as D
-    from oracle import kv as OK
-    from oracle.shape import KVShape
     world = 1 if dist is None else dist.world
     rank = 0 if dist is None else dist.rank
     device = 0 if dist is None else dist.device
@@ -836,7 +813,7 @@ def c5_leg(aeg, torch, kernel, dist=None, tp_rank=1, tp_size=4, reps=3, model="q
         tp_rank = rank % (world // 2)
     seed_w, seed_kv = gi.w_seed(5), gi.kv_seed(5)
     sht = gi.KV_SHAPES["qwen-72b-tp4"]
-    sh = KVShape(*sht)
+    sh = aeg.KVShape.of(sht)
     n_kv = (2 * GIB) // sh.block_bytes()
     slab = 10 * 64 * MIB * 2            # 1.25 GiB: 128 blocks of 10 MiB
     nslab = -(-n_kv // (slab // sh.block_bytes())) + 1
@@ -859,8 +836,6 @@ def c5_leg(aeg, torch, kernel, dist=None, tp_rank=1, tp_size=4, reps=3, model="q
     if prefill:
         a = aeg.Context(device, aeg.default_config(device_kv_bytes=nslab * slab, host_kv_bytes=GIB, dev_slab_bytes=slab,
                                                    dev_slab_layout=aeg.LAYER_MAJOR, kernel=kernel, flags=aeg.CFG_TIMING))
-    geom_a = OK.PoolGeom(nslab * slab, slab, aeg.LAYER_MAJOR)
-    geom_b = OK.PoolGeom(nslab * slab, slab, aeg.BLOCK_MAJOR)
     # pools + destination handles
     if world == 1:
         a.import_peer(1, b.export_ipc())
@@ -878,9 +853,8 @@ def c5_leg(aeg, torch, kernel, dist=None, tp_rank=1, tp_size=4, reps=3, model="q
     if prefill:
         src = a.kv_alloc(0, sht, n_kv)
         abase, _ = a.pool_region(0)
-        so = [aeg.decode_block(x)[1:] for x in src]
-        D.fill_chunks(abase, [OK.addr(geom_a, sh, h, l) for h in so for l in range(sh.L)],
-                      [gi.kv_key(5, rank, i, l) for i in range(n_kv) for l in range(sh.L)], sh.chunk_bytes(), seed_kv)
+        D.fill_chunks(abase, chunk_offsets(a, 0, sht, src),
+                      [gi.kv_key(5, rank, i, l) for i in range(n_kv) for l in range(sh.num_layers)], sh.chunk_bytes(), seed_kv)
     dst_handles = dst if world == 1 else (dst_by_rank.get(rank + world // 2) if prefill else None)
     D.sync()
 
@@ -922,14 +896,13 @@ def c5_leg(aeg, torch, kernel, dist=None, tp_rank=1, tp_size=4, reps=3, model="q
         offs, x = b.weights_stage(descs, tp_rank, tp_size)
         b.layer_ready(x, -1, aeg.READY_BLOCK)
         b.xfer_release(x)
-        w_ok, picks = _c5_check_weights(aeg, b, model, 7, seed_w, tp_rank, tp_size, offs, pick)
+        w_ok, picks = (check or _c5_check_weights)(aeg, b, model, 7, seed_w, tp_rank, tp_size, offs, pick)
     kv_bad = 0
     if decode:
         sender = 0 if world == 1 else rank - world // 2
         bbase, _ = b.pool_region(0)
-        do = [aeg.decode_block(x)[1:] for x in dst]
-        kv_bad, _ = D.verify_chunks(bbase, [OK.addr(geom_b, sh, h, l) for h in do for l in range(sh.L)],
-                                    [gi.kv_key(5, sender, i, l) for i in range(n_kv) for l in range(sh.L)],
+        kv_bad, _ = D.verify_chunks(bbase, chunk_offsets(b, 0, sht, dst),
+                                    [gi.kv_key(5, sender, i, l) for i in range(n_kv) for l in range(sh.num_layers)],
                                     sh.chunk_bytes(), seed_kv)
     shard = 0 if not decode else sum(d["rows"] * d["cols"] * 2 // (1 if d["split"] == gi.REPLICATED else tp_size)
                                      for d in descs)
@@ -1188,41 +1161,52 @@ def run_ours(args):
                    "h2d_bytes_per_step": int(bytes_step // 2 + 2 * sb.n * 8),
                    "d2h_bytes_per_step": int(bytes_step // 2),
                    "how": "wall clock around the Python-API calls of one step incl. host sync"}
-        one_dir = sb.one_direction(torch, cons)
-        ver = sb.replay_and_verify()
+        def leg(name, fn):
+            """A side leg that fails reports its error in the line instead of losing the whole line."""
+            try:
+                return fn()
+            except Exception as e:  # noqa: BLE001
+                import traceback
+                log(f"[rank {rank}] leg {name} failed:\n" + traceback.format_exc())
+                return {"error": f"{type(e).__name__}: {e}"}
+
+        one_dir = leg("one_direction", lambda: sb.one_direction(torch, cons))
+        ver = leg("verify", sb.verify)
         if world > 1:   # every rank checks its own pools; the line reports all of them
-            ver["ranks_failed"] = int(dist.sum(0 if ver["ok"] else 1))
+            ver["ranks_failed"] = int(dist.sum(0 if ver.get("ok") else 1))
             ver["ok"] = ver["ranks_failed"] == 0
         sb.ctx.shutdown()
         if args.no_migrate:
             mig = None
         elif world > 1:
-            mig = migrate_leg_dist(aeg, torch, dist, kernel)
+            mig = leg("migrate", lambda: migrate_leg_dist(aeg, torch, dist, kernel))
         else:
-            mig = migrate_leg(aeg, torch, kernel)
+            mig = leg("migrate", lambda: migrate_leg(aeg, torch, kernel))
         sw = None
         if not (args.no_switch or world > 1):
             t0 = time.time()
             descs, caches = model_caches(["qwen-1.8b", "llama-7b", "yi-9b"])
             gen_s = time.time() - t0
-            sw = {"staged": switch_leg(aeg, torch, args.switches, kernel, descs, "staged"),
-                  "prefetch": switch_leg(aeg, torch, args.switches, kernel, descs, "prefetch"),
-                  "direct": switch_leg(aeg, torch, args.switches, kernel, descs, "direct", caches),
+            sw = {"staged": leg("switch_staged", lambda: switch_leg(aeg, torch, args.switches, kernel, descs, "staged")),
+                  "prefetch": leg("switch_prefetch",
+                                  lambda: switch_leg(aeg, torch, args.switches, kernel, descs, "prefetch")),
+                  "direct": leg("switch_direct",
+                                lambda: switch_leg(aeg, torch, args.switches, kernel, descs, "direct", caches)),
                   "model_cache_gen_s": round(gen_s, 1)}
             del caches
-        ovl = None if args.no_switch or world > 1 else overlap_leg(aeg, torch, kernel)
+        ovl = None if args.no_switch or world > 1 else leg("overlap", lambda: overlap_leg(aeg, torch, kernel))
         if args.no_c5:
             c5 = None
         elif world in (1, 8):
-            c5 = c5_leg(aeg, torch, kernel, dist if world > 1 else None, model=args.c5_model)
+            c5 = leg("c5", lambda: c5_leg(aeg, torch, kernel, dist if world > 1 else None, model=args.c5_model))
         else:
             c5 = {"skipped": "configs[4] is the 8-GPU TP=4 layout (one rank pair on 1 GPU); not defined for N=%d" % world}
-        alloc = allocator_leg(aeg) if rank == 0 else None
-        cpu = None if args.no_cpu or rank != 0 else cpu_baseline()
+        alloc = leg("allocator", lambda: allocator_leg(aeg)) if rank == 0 else None
+        cpu = None if args.no_cpu or rank != 0 else leg("cpu_baseline", cpu_baseline)
         out.update({"e2e": e2e, "verify": ver, "one_direction": one_dir, "pcie_memcpy_GBps": {k: round(v, 1) for k, v in pc.items()},
                     "switch": sw, "migrate": mig, "per_layer_overlap": ovl, "c5": c5, "allocator": alloc,
                     "cpu_baseline": cpu})
-        if not ver["ok"]:
+        if not ver.get("ok"):
             log("VERIFICATION FAILED", ver)
     else:
         sb.ctx.shutdown()
@@ -1249,11 +1233,11 @@ def run_ours(args):
                      "frac_of_duplex_nominal": round(bytes_step / (ms_step * 1e6) / (2 * PCIE_NOMINAL), 3)},
             "clocks": clocks,
             "gpu_launches": launches_all,
-            "consumer_launches": args.steps * sb.sh.L,
+            "consumer_launches": args.steps * sb.L,
         }
         res.update(out)
         od = out.get("one_direction")
-        if od:   # each direction alone against PCIe Gen5 x16 nominal 64 GB/s (target >= 0.80)
+        if od and "error" not in od:   # each direction alone against PCIe Gen5 x16 nominal 64 GB/s (target >= 0.80)
             res["pcie"]["swap_out_alone_GBps"] = od["swap_out"]["GBps"]
             res["pcie"]["swap_in_alone_GBps"] = od["swap_in"]["GBps"]
             res["pcie"]["swap_out_alone_frac"] = round(od["swap_out"]["GBps"] / PCIE_NOMINAL, 3)

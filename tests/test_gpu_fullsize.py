@@ -21,15 +21,18 @@ def test_c2_full_size_round_trip():
     require_gpu()
     import torch
     import bench
-    sb = bench.SwapBench(aeg, bench.QWEN7B, 64, aeg.KERNEL_AUTO).setup()
+    from .oracle_swapbench import OracleSwapBench
+    sb = OracleSwapBench(aeg, bench.QWEN7B, 64, aeg.KERNEL_AUTO).setup()
     try:
         sb.sink = torch.zeros(1, dtype=torch.int64, device="cuda")
         cons = torch.cuda.Stream()
         sb.step(torch, cons)
-        sb.step(torch, cons, with_consumer=False)
+        sb.step(torch, cons, with_consumer=False, keep_host_offsets=True)
         v = sb.replay_and_verify()
         assert v["device_chunks_checked"] > 300_000 and v["host_chunks_checked"] >= sb.n * 32
         assert v["ok"], v
+        w = sb.verify()   # bench.py's own (oracle-free) invariant check agrees
+        assert w["ok"] and w["batch_host_chunks_checked"] == sb.n * 32, w
     finally:
         sb.ctx.shutdown()
 
