@@ -65,6 +65,7 @@ def parse():
     # exercise knobs (several ranks sharing one GPU): not used for reported numbers
     p.add_argument("--c5-model", default="qwen-72b", help=argparse.SUPPRESS)
     p.add_argument("--churn-slabs", type=int, default=12, help=argparse.SUPPRESS)
+    p.add_argument("--migrate-requests", type=int, default=16, help=argparse.SUPPRESS)
     p.add_argument("--no-e2e", action="store_true")
     p.add_argument("--no-cpu", action="store_true")
     p.add_argument("--switches", type=int, default=30)
@@ -587,7 +588,7 @@ def switch_leg(aeg, torch, n_switch, kernel, descs, mode="staged", caches=None):
                                 "fill_wait_slot_ms": round(wslot, 1)}}
 
 
-def migrate_leg(aeg, torch, kernel, n_req=4):
+def migrate_leg(aeg, torch, kernel, n_req=16, src_layout=None, dst_layout=None):
     """configs[2] shapes on one GPU: Llama-2-13B KV hand-off through the fused migrate kernel into
     another context's pool (peer mapped in-process, the same kernel that stores over NVLink when the
     peer is another GPU).  Checked against the generator at the destination blocks' chunks (identity
@@ -603,7 +604,8 @@ def migrate_leg(aeg, torch, kernel, n_req=4):
     mk = lambda lay: aeg.Context(0, aeg.default_config(device_kv_bytes=nslab * slab, host_kv_bytes=GIB,  # noqa: E731
                                                        dev_slab_bytes=slab, dev_slab_layout=lay, kernel=kernel,
                                                        flags=aeg.CFG_TIMING))
-    a, b = mk(aeg.LAYER_MAJOR), mk(aeg.BLOCK_MAJOR)
+    a = mk(aeg.LAYER_MAJOR if src_layout is None else src_layout)
+    b = mk(aeg.BLOCK_MAJOR if dst_layout is None else dst_layout)
     sc = a.kv_alloc(0, sht, n)
     dc = b.kv_alloc(0, sht, n)
     abase, _ = a.pool_region(0)
@@ -641,7 +643,7 @@ def migrate_leg(aeg, torch, kernel, n_req=4):
             "kernel_ms_per_xfer": round(kms, 3), "bit_exact": bad == 0}
 
 
-def migrate_leg_dist(aeg, torch, dist, kernel, n_req=4):
+def migrate_leg_dist(aeg, torch, dist, kernel, n_req=16):
     """configs[2] across GPUs: prefill rank i hands n_req Llama-2-13B-shaped requests to decode rank
     i + N/2 over NVLink/NVSwitch (fused gather -> remote 16-byte stores), per-layer IPC events.
     Aggregate GB/s = all pairs' payload / max-over-ranks device time."""
@@ -1179,9 +1181,9 @@ def run_ours(args):
         if args.no_migrate:
             mig = None
         elif world > 1:
-            mig = leg("migrate", lambda: migrate_leg_dist(aeg, torch, dist, kernel))
+            mig = leg("migrate", lambda: migrate_leg_dist(aeg, torch, dist, kernel, args.migrate_requests))
         else:
-            mig = leg("migrate", lambda: migrate_leg(aeg, torch, kernel))
+            mig = leg("migrate", lambda: migrate_leg(aeg, torch, kernel, args.migrate_requests))
         sw = None
         if not (args.no_switch or world > 1):
             t0 = time.time()
