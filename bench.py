@@ -1125,15 +1125,19 @@ def run_ours(args):
     dist.barrier()
     with Clocks(dist.device) as clk:
         e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        marks = [torch.cuda.Event(enable_timing=True) for _ in range(args.steps)]
         e0.record(cons)
-        for _ in range(args.steps):
+        for i in range(args.steps):
             sb.step(torch, cons)
+            marks[i].record(cons)
         e1.record(cons)
         e1.synchronize()
     dist.barrier()
     ms_total = dist.max(e0.elapsed_time(e1))
     clocks = clk.summary()
     ms_step = ms_total / args.steps
+    per_step = sorted(dist.max(a.elapsed_time(b)) for a, b in zip([e0] + marks[:-1], marks))
+    pct = lambda q: round(per_step[min(len(per_step) - 1, int(q * (len(per_step) - 1) + 0.5))], 2)  # noqa: E731
     total_bytes = dist.sum(bytes_step * args.steps)
     value = total_bytes / (ms_total * 1e6)
     g = sb.ctx.kernel_stats(aeg.K_GATHER)
@@ -1215,7 +1219,8 @@ def run_ours(args):
     if rank == 0:
         res = {
             "metric": METRIC, "value": round(value, 2), "unit": "GB/s", "n_gpus": world, "steps": args.steps,
-            "warmup": args.warmup, "ms_per_step": round(ms_step, 2), "higher_is_better": True, "scaling": "weak",
+            "warmup": args.warmup, "ms_per_step": round(ms_step, 2),
+            "step_ms_p10_p50_p90": [pct(0.1), pct(0.5), pct(0.9)], "higher_is_better": True, "scaling": "weak",
             "vs_baseline": None, "dtype": "u8", "data": "synthetic",
             "config": {"workload": "configs[1]: Qwen-7B-shaped KV (32 layers, 32 KV heads, d=128, bf16, 16-token "
                                    f"blocks), {n_req}-request decode batch swapped out and back in per step",
