@@ -213,6 +213,20 @@ int aegin_copy(void* dst, const void* src, uint64_t n) { return int(cudaMemcpy(d
 
 int aegin_sync(void) { return int(cudaDeviceSynchronize()); }
 
+// Baseline for the bench (what the paper's "memcpy(async)" per block amounts to for paged KV): one
+// cudaMemcpyAsync per chunk, dst_base + dst_off[i] <- src_base + src_off[i], on `stream`
+// (copy engines; host or device pointers, UVA).
+int aegin_copy_chunks(void* dst_base, const uint64_t* dst_off, const void* src_base, const uint64_t* src_off,
+                      uint64_t n, uint64_t chunk, void* stream) {
+  for (uint64_t i = 0; i < n; ++i) {
+    cudaError_t e = cudaMemcpyAsync(static_cast<char*>(dst_base) + dst_off[i],
+                                    static_cast<const char*>(src_base) + src_off[i], chunk, cudaMemcpyDefault,
+                                    static_cast<cudaStream_t>(stream));
+    if (e != cudaSuccess) return int(e);
+  }
+  return 0;
+}
+
 // Load every kernel of this library now (no lazy module load later, which would wait for a
 // running gate kernel and deadlock a race test).
 int aegin_preload(void) {

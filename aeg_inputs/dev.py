@@ -33,6 +33,7 @@ def lib():
             "aegin_sync": [],
             "aegin_host_fill": [P, U64, U64, U64, C.c_int],
             "aegin_host_fill_2d": [P, U64, U64, U64, U64, U64, C.c_int],
+            "aegin_copy_chunks": [P, PU64, P, PU64, U64, U64, P],
         }
         for k, a in sig.items():
             getattr(L, k).argtypes = a
@@ -127,3 +128,10 @@ def host_fill_2d(ptr: int, rows: int, pitch: int, width: int, seed: int, key: in
     """Fill `rows` runs of `width` bytes at `pitch` from `ptr` with the bytes a dense host_fill of
     the [rows x pitch] region (key base `key`) would put there."""
     _ck(lib().aegin_host_fill_2d(P(ptr), rows, pitch, width, seed, key, threads))
+
+
+def copy_chunks(dst_base: int, dst_offs, src_base: int, src_offs, chunk: int, stream: int = 0):
+    """One cudaMemcpyAsync per chunk (the per-block memcpy baseline)."""
+    d, s_ = _u64(dst_offs), _u64(src_offs)
+    _ck(lib().aegin_copy_chunks(P(dst_base), d.ctypes.data_as(PU64), P(src_base), s_.ctypes.data_as(PU64), d.size,
+                                chunk, P(stream)))

@@ -396,6 +396,89 @@ class SwapBench:
 
 
 # ----------------------------------------------------------------------------------- legs
+def chunk_memcpy_baseline(aeg, torch, ctx, sht, src_blocks, reps=2):
+    """The per-block memcpy the paper's swap amounts to for paged KV ("memcpy(async)"
+    Fig. 10; vLLM-style swap_blocks): one cudaMemcpyAsync per (block, layer) chunk, device blocks ->
+    host blocks, then host -> fresh device blocks, on one stream (copy engines only).  Same blocks and
+    placement as the library's swap; timed with CUDA events.  Returns GB/s per direction."""
+    from aeg_inputs import dev as D
+    sh = aeg.KVShape.of(sht)
+    n = len(src_blocks)
+    hc = ctx.kv_alloc(aeg.POOL_HOST, sht, n)
+    nd = ctx.kv_alloc(aeg.POOL_DEVICE, sht, n)
+    dbase, _ = ctx.pool_region(aeg.POOL_DEVICE)
+    hbase, _ = ctx.pool_region(aeg.POOL_HOST)
+    so, ho, no = (chunk_offsets(ctx, p, sht, b) for p, b in ((0, src_blocks), (1, hc), (0, nd)))
+    s = torch.cuda.Stream()
+    out = {}
+    for name, args in (("d2h", (hbase, ho, dbase, so)), ("h2d", (dbase, no, hbase, ho))):
+        ts = []
+        for _ in range(reps):
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record(s)
+            D.copy_chunks(*args, sh.chunk_bytes(), s.cuda_stream)
+            e1.record(s)
+            e1.synchronize()
+            ts.append(e0.elapsed_time(e1))
+        out[name + "_GBps"] = round(n * sh.block_bytes() / (min(ts) * 1e6), 2)
+    out["memcpy_calls_per_direction"] = int(so.size)
+    out["chunk_bytes"] = sh.chunk_bytes()
+    ctx.kv_free(aeg.POOL_HOST, hc)
+    ctx.kv_free(aeg.POOL_DEVICE, nd)
+    return out
+
+
+def small_chunk_leg(aeg, torch, kernel, model="yi-9b", gib=1):
+    """Swap-out / swap-in of `gib` GiB of a small-chunk KV shape (Yi-9B: 48 layers x 32 KiB chunks,
+    the configs[3] model with the smallest chunk) through the library, next to the per-chunk memcpy
+    baseline on the same blocks.  Correctness: the round trip is the identity on every chunk."""
+    import aeg_inputs as gi
+    from aeg_inputs import dev as D
+    sht = gi.KV_SHAPES[model]
+    sh = aeg.KVShape.of(sht)
+    n = (gib * GIB) // sh.block_bytes()
+    ctx = aeg.Context(0, aeg.default_config(device_kv_bytes=3 * gib * GIB + GIB, host_kv_bytes=gib * GIB + GIB,
+                                            kernel=kernel, flags=aeg.CFG_TIMING))
+    dbase, _ = ctx.pool_region(0)
+    hbase, _ = ctx.pool_region(1)
+    src = ctx.kv_alloc(0, sht, n)
+    keys = np.array([gi.kv_key(3, 0, i, l) for i in range(n) for l in range(sh.num_layers)], np.uint64)
+    seed = gi.kv_seed(4)
+    D.fill_chunks(dbase, chunk_offsets(ctx, 0, sht, src), keys, sh.chunk_bytes(), seed)
+    s = torch.cuda.Stream()
+    res = {}
+    for it in range(3):
+        hc = ctx.kv_alloc(1, sht, n)
+        nd = ctx.kv_alloc(0, sht, n)
+        ms = []
+        for kind in ("out", "in"):
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record(s)
+            ctx.stream_fence(s.cuda_stream)
+            x = ctx.kv_swap_out(sht, src, hc, flags=aeg.FREE_SRC) if kind == "out" else \
+                ctx.kv_swap_in(sht, hc, nd, flags=aeg.FREE_SRC)
+            ctx.layer_ready(x, -1, aeg.READY_WAIT_STREAM, s.cuda_stream)
+            e1.record(s)
+            e1.synchronize()
+            ctx.layer_ready(x, -1, aeg.READY_BLOCK)
+            ctx.xfer_release(x)
+            ms.append(e0.elapsed_time(e1))
+        src = nd
+        if it > 0:
+            res.setdefault("out", []).append(ms[0])
+            res.setdefault("in", []).append(ms[1])
+    bad, _ = D.verify_chunks(dbase, chunk_offsets(ctx, 0, sht, src), keys, sh.chunk_bytes(), seed)
+    ctx.reclaim(True)
+    base = chunk_memcpy_baseline(aeg, torch, ctx, sht, src)
+    ctx.shutdown()
+    b = n * sh.block_bytes()
+    return {"workload": f"{model} KV ({n} blocks x {sh.num_layers} layers, {sh.chunk_bytes() >> 10} KiB chunks, "
+                        f"{b / GIB:.2f} GiB) swap-out and swap-in, each alone",
+            "swap_out_GBps": round(b / (min(res["out"]) * 1e6), 2), "swap_in_GBps": round(b / (min(res["in"]) * 1e6), 2),
+            "per_chunk_memcpy": base, "bit_exact": bad == 0}
+
+
+
 def pcie_calibration(torch):
     """Plain cudaMemcpy of 1 GiB pinned <-> device: the copy engines' measured ceiling here."""
     h = torch.empty(GIB, dtype=torch.uint8, pin_memory=True)
@@ -1178,6 +1261,7 @@ def run_ours(args):
 
         one_dir = leg("one_direction", lambda: sb.one_direction(torch, cons))
         ver = leg("verify", sb.verify)
+        base = leg("memcpy_baseline", lambda: chunk_memcpy_baseline(aeg, torch, sb.ctx, sb.sht, sb.src_c))
         if world > 1:   # every rank checks its own pools; the line reports all of them
             ver["ranks_failed"] = int(dist.sum(0 if ver.get("ok") else 1))
             ver["ok"] = ver["ranks_failed"] == 0
@@ -1207,10 +1291,12 @@ def run_ours(args):
             c5 = leg("c5", lambda: c5_leg(aeg, torch, kernel, dist if world > 1 else None, model=args.c5_model))
         else:
             c5 = {"skipped": "configs[4] is the 8-GPU TP=4 layout (one rank pair on 1 GPU); not defined for N=%d" % world}
+        small = None if world > 1 else leg("small_chunk", lambda: small_chunk_leg(aeg, torch, kernel))
         alloc = leg("allocator", lambda: allocator_leg(aeg)) if rank == 0 else None
         cpu = None if args.no_cpu or rank != 0 else leg("cpu_baseline", cpu_baseline)
         out.update({"e2e": e2e, "verify": ver, "one_direction": one_dir, "pcie_memcpy_GBps": {k: round(v, 1) for k, v in pc.items()},
                     "switch": sw, "migrate": mig, "per_layer_overlap": ovl, "c5": c5, "allocator": alloc,
+                    "per_chunk_memcpy_baseline": base, "small_chunk": small,
                     "cpu_baseline": cpu})
         if not ver.get("ok"):
             log("VERIFICATION FAILED", ver)

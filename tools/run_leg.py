@@ -15,5 +15,6 @@ build.build()
 leg = sys.argv[1]
 kernel = {"auto": aeg.KERNEL_AUTO, "lsu": aeg.KERNEL_LSU, "bulk": aeg.KERNEL_BULK}[sys.argv[2] if len(sys.argv) > 2 else "auto"]
 fn = {"c5": lambda: bench.c5_leg(aeg, torch, kernel), "migrate": lambda: bench.migrate_leg(aeg, torch, kernel),
-      "overlap": lambda: bench.overlap_leg(aeg, torch, kernel)}[leg]
+      "overlap": lambda: bench.overlap_leg(aeg, torch, kernel),
+      "small_chunk": lambda: bench.small_chunk_leg(aeg, torch, kernel)}[leg]
 print(json.dumps(fn()), flush=True)
