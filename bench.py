@@ -715,6 +715,16 @@ def migrate_leg(aeg, torch, kernel, n_req=16, src_layout=None, dst_layout=None):
     nl, nbytes, kms = a.kernel_stats(aeg.K_MIGRATE)
     doffs = chunk_offsets(b, 0, sht, dc)
     bad, _ = D.verify_chunks(bbase, doffs, keys, sh.chunk_bytes(), seed)
+    # baseline on the same blocks: one cudaMemcpyAsync (copy engine, D2D) per (block, layer) chunk
+    s = torch.cuda.Stream()
+    bt = []
+    for _ in range(2):
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(s)
+        D.copy_chunks(bbase, doffs, abase, offs, sh.chunk_bytes(), s.cuda_stream)
+        e1.record(s)
+        e1.synchronize()
+        bt.append(e0.elapsed_time(e1))
     a.shutdown()
     b.shutdown()
     payload = n * sh.block_bytes()
@@ -723,7 +733,9 @@ def migrate_leg(aeg, torch, kernel, n_req=16, src_layout=None, dst_layout=None):
                         "in-process; NVLink path needs >= 2 GPUs)",
             "payload_bytes": payload, "ms": round(ms, 3), "GBps_payload": round(payload / (ms * 1e6), 1),
             "hbm_GBps": round(2 * payload / (ms * 1e6), 1), "kernel_launches_per_xfer": nl,
-            "kernel_ms_per_xfer": round(kms, 3), "bit_exact": bad == 0}
+            "kernel_ms_per_xfer": round(kms, 3), "bit_exact": bad == 0,
+            "per_chunk_memcpy_baseline_GBps_payload": round(payload / (min(bt) * 1e6), 1),
+            "per_chunk_memcpy_calls": int(len(offs))}
 
 
 def migrate_leg_dist(aeg, torch, dist, kernel, n_req=16):
