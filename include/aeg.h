@@ -81,7 +81,9 @@ enum {
   AEG_CFG_SHARED_HOST = 1u << 3 /* CPU KV region in POSIX shared memory, mappable by peers:
                                    the node-shared "Unified CPU KV Cache" (Fig. 5) */
 };
-/* kernel selection for gather/scatter/migrate (AEG_KERNEL_AUTO picks the measured best) */
+/* kernel selection for gather/scatter/migrate.  AEG_KERNEL_AUTO picks the measured best by chunk
+ * size Cl: gather/scatter WARP if Cl <= 4 KiB, LSU if Cl < 64 KiB, BULK otherwise;
+ * migrate (paged -> paged, local or peer) WARP if Cl <= 4 KiB, LSU otherwise. */
 enum { AEG_KERNEL_AUTO = 0, AEG_KERNEL_LSU = 1, AEG_KERNEL_BULK = 2, AEG_KERNEL_WARP = 3 };
 
 /* ---- structs ---------------------------------------------------------------------------- */
@@ -145,7 +147,7 @@ typedef struct {
 /* ---- lifecycle -------------------------------------------------------------------------- */
 
 /* Fill *cfg with defaults: 1 GiB slabs (layer-major), 2 GiB stage ring of 64 MiB chunks,
- * 3 x 1 GiB staging slots per direction, 8 host threads, AUTO kernels (BULK); region sizes 0.
+ * 3 x 1 GiB staging slots per direction, 8 host threads, AUTO kernels; region sizes 0.
  * Returns AEG_OK. */
 int aeg_config_default(aeg_config* cfg);
 
