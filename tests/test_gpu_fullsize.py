@@ -65,3 +65,64 @@ def test_qwen18b_tp2_weights_full_size_sampled():
             assert np.array_equal(got, sh), (k, d["name"])
     finally:
         ctx.shutdown()
+
+
+def test_c3_full_size_handoff():
+    """configs[2] at the size bench.py times on one GPU: 16 Llama-2-13B requests (2,346 blocks,
+    30.7 GB) from a layer-major pool into a block-major pool of another context (peer-mapped), AUTO
+    kernel (LSU).  Expected image: oracle O7 on chunk labels over the whole destination pool
+    (every chunk, including the untouched poison around the destination blocks)."""
+    require_gpu()
+    from oracle import kv as OK
+    from oracle.shape import KVShape
+    from oracle.slab import SlabPool
+    sht = gi.KV_SHAPES["llama-2-13b"]
+    sh = KVShape(*sht)
+    cl = sh.chunk_bytes()
+    lens = gi.request_lengths(3, 16, 512, 4096)
+    blocks = [-(-t // 16) for t in lens]
+    n = sum(blocks)
+    slab = (1 << 30) + (256 << 20)
+    nslab = -(-n // (slab // sh.block_bytes())) + 1
+    seed = gi.kv_seed(3)
+    mk = lambda lay: aeg.Context(0, aeg.default_config(device_kv_bytes=nslab * slab, host_kv_bytes=1 << 30,  # noqa: E731
+                                                       dev_slab_bytes=slab, dev_slab_layout=lay))
+    a, b = mk(aeg.LAYER_MAJOR), mk(aeg.BLOCK_MAJOR)
+    try:
+        ga = OK.PoolGeom(nslab * slab, slab, aeg.LAYER_MAJOR)
+        gb = OK.PoolGeom(nslab * slab, slab, aeg.BLOCK_MAJOR)
+        oa, ob = SlabPool(ga.nbytes, slab), SlabPool(gb.nbytes, slab)
+        abase, _ = a.pool_region(0)
+        bbase, _ = b.pool_region(0)
+        D.fill_region(bbase, gb.nbytes, seed, gi.poison_key(gi.TAG_NEVER, 0))
+        cells = gb.nbytes // cl
+        blab = np.uint64(gi.poison_key(gi.TAG_NEVER, 0)) + np.arange(cells, dtype=np.uint64) * np.uint64(cl // 8)
+        alab = np.zeros(ga.nbytes // cl, dtype=np.uint64)
+        sc, so = a.kv_alloc(0, sht, n), oa.alloc(sh, n)
+        dc, do = b.kv_alloc(0, sht, n), ob.alloc(sh, n)
+        assert [aeg.decode_block(x)[1:] for x in sc] == list(so)
+        assert [aeg.decode_block(x)[1:] for x in dc] == list(do)
+        labels = [(r, j) for r, k in enumerate(blocks) for j in range(k)]
+        offs = np.array([OK.addr(ga, sh, h, l) for h in so for l in range(sh.L)], np.uint64)
+        keys = np.array([gi.kv_key(1, r, j, l) for (r, j) in labels for l in range(sh.L)], np.uint64)
+        for i in range(0, offs.size, 1 << 16):
+            D.fill_chunks(abase, offs[i:i + (1 << 16)], keys[i:i + (1 << 16)], cl, seed)
+        alab[(offs // np.uint64(cl)).astype(np.int64)] = keys
+        a.import_peer(1, b.export_ipc())
+        x = a.kv_migrate(sht, sc, 1, dc)
+        a.layer_ready(x, -1, aeg.READY_BLOCK)
+        a.xfer_release(x)
+        exp = OK.migrate(alab, ga, blab, gb, sh, so, do, unit=cl)
+        bad = 0
+        allo = np.arange(cells, dtype=np.uint64) * np.uint64(cl)
+        for i in range(0, cells, 1 << 16):
+            bd, _ = D.verify_chunks(bbase, allo[i:i + (1 << 16)], exp[i:i + (1 << 16)], cl, seed)
+            bad += bd
+        assert bad == 0
+        # two chunks byte-for-byte against the NumPy generator
+        for h, l in ((do[0], 0), (do[-1], sh.L - 1)):
+            o = OK.addr(gb, sh, h, l)
+            assert np.array_equal(D.read(bbase + o, cl), gi.region_bytes(seed, int(exp[o // cl]), cl))
+    finally:
+        a.shutdown()
+        b.shutdown()
