@@ -517,7 +517,7 @@ def model_caches(names):
     return descs, caches
 
 
-def switch_leg(aeg, torch, n_switch, kernel, descs, mode="staged", caches=None):
+def switch_leg(aeg, torch, n_switch, kernel, descs, mode="staged", caches=None, kv_out="after"):
     """configs[3]: token-level switch among Qwen-1.8B / Llama-7B / Yi-9B shapes on one GPU.
     staged  : switch(A->B) = swap-out of A's 1 GiB decode KV (D2H) || staging of B's weights through
               the pinned Stage Buffer (H2D, Fig. 9 3.a) -> swap-in of B's KV.
@@ -571,9 +571,13 @@ def switch_leg(aeg, torch, n_switch, kernel, descs, mode="staged", caches=None):
         e0 = torch.cuda.Event(enable_timing=True)
         e0.record(cons)
         ctx.stream_fence(cons.cuda_stream)
-        hb = ctx.kv_alloc(aeg.POOL_HOST, shapes[cur], kv[cur][1])
-        xo = ctx.kv_swap_out(shapes[cur], kv[cur][0], hb, flags=aeg.FREE_SRC)        # A's KV out (D2H)
-        kv[cur] = (hb, kv[cur][1])
+
+        def a_kv_out(a=cur):                                                           # A's KV out (D2H)
+            hb = ctx.kv_alloc(aeg.POOL_HOST, shapes[a], kv[a][1])
+            x = ctx.kv_swap_out(shapes[a], kv[a][0], hb, flags=aeg.FREE_SRC)
+            kv[a] = (hb, kv[a][1])
+            return x
+        xo = a_kv_out() if kv_out == "concurrent" else None
         # B's KV goes first: the copy engine serves one busy H2D stream until it drains
         # (profiles/r01/ce_probe.txt), so KV queued behind a model's weights would land last
         nsh = shapes[nxt]
@@ -593,9 +597,11 @@ def switch_leg(aeg, torch, n_switch, kernel, descs, mode="staged", caches=None):
         diag = {}
         if i == 3:   # one switch: when does each piece land (device timeline, separate streams)?
             # KV probes first: a weights-layer wait blocks the host until the pipeline records it
-            for name, (xx, l) in {"kv_l0": (xi, 0), "kv_last": (xi, nsh[0] - 1), "kv_out_all": (xo, -1),
-                                  "weights_l0": (xw, wl(0)), "weights_l1": (xw, wl(1)), "weights_all": (xw, -1)
-                                  }.items():
+            probes = {"kv_l0": (xi, 0), "kv_last": (xi, nsh[0] - 1), "kv_out_all": (xo, -1),
+                      "weights_l0": (xw, wl(0)), "weights_l1": (xw, wl(1)), "weights_all": (xw, -1)}
+            if xo is None:
+                del probes["kv_out_all"]
+            for name, (xx, l) in probes.items():
                 ds = torch.cuda.Stream()
                 ctx.layer_ready(xx, l, aeg.READY_WAIT_STREAM, ds.cuda_stream)
                 de = torch.cuda.Event(enable_timing=True)
@@ -613,6 +619,18 @@ def switch_leg(aeg, torch, n_switch, kernel, descs, mode="staged", caches=None):
         ctx.layer_ready(xw, -1, aeg.READY_WAIT_STREAM, cons.cuda_stream)
         e_end = torch.cuda.Event(enable_timing=True)
         e_end.record(cons)
+        if xo is None:
+            # PCIe duplex costs each direction ~10 % here (bidirectional memcpy ~99 GB/s total vs
+            # 55-57 one way), so A's KV-out waits until B has landed and overlaps B's decode
+            # instead of B's load (ordered after the consumer stream: aeg_stream_fence)
+            ctx.stream_fence(cons.cuda_stream)
+            xo = a_kv_out()
+            if diag:
+                ds = torch.cuda.Stream()
+                ctx.layer_ready(xo, -1, aeg.READY_WAIT_STREAM, ds.cuda_stream)
+                de = torch.cuda.Event(enable_timing=True)
+                de.record(ds)
+                diag["kv_out_all"] = de
         e_end.synchronize()
         for xx in (xo, xw, xi):
             ctx.layer_ready(xx, -1, aeg.READY_BLOCK)
@@ -664,7 +682,8 @@ def switch_leg(aeg, torch, n_switch, kernel, descs, mode="staged", caches=None):
     how = {"staged": "weights staged through the 2 GiB pinned Stage Buffer by host threads (3.a)",
            "direct": "weights DMA'd straight from the page-locked Model Cache (registered once)",
            "prefetch": "weights prefetched during the previous turn, relocated on-device at the switch (3.b)"}[mode]
-    return {"workload": f"configs[3] 3-model switch (Qwen-1.8B, Llama-7B, Yi-9B shapes), 1 GiB KV each; {how}",
+    return {"workload": f"configs[3] 3-model switch (Qwen-1.8B, Llama-7B, Yi-9B shapes), 1 GiB KV each; {how}; "
+                        f"A's KV out {'after B has landed' if kv_out == 'after' else 'concurrent with B loading'}",
             "per_model": per, "weights_bit_exact_sample": bad == 0, "register_s": reg_s,
             "landing_ms_one_switch": diag_ms,
             "weight_pipeline": {"chunks": wchunks, "issuer_wait_fill_ms": round(wfill, 1),
