@@ -819,7 +819,10 @@ def migrate_leg_dist(aeg, torch, dist, kernel, n_req=16):
             ctx.xfer_release(x)
         return dist.max(ms)
 
+    ctx.kernel_stats_reset()
     times = [hand_off(pairs) for _ in range(5)][1:]
+    kl, kb, kms = ctx.kernel_stats(aeg.K_MIGRATE)   # prefill ranks: 5 rounds of migrate launches
+    k_gbps = dist.max(kb / 2 / (kms * 1e6) if kms > 0 else 0.0)   # payload bytes over the link
     bad = 0
     if not prefill:
         sender = [s_ for s_, d in pairs if d == rank][0]
@@ -840,6 +843,8 @@ def migrate_leg_dist(aeg, torch, dist, kernel, n_req=16):
     return {"workload": f"configs[2] Llama-2-13B hand-off, {n_req} requests per pair, pairs {pairs}",
             "payload_bytes": payload, "ms": round(ms, 3), "GBps_aggregate": round(payload / (ms * 1e6), 1),
             "GBps_per_pair": round(payload / len(pairs) / (ms * 1e6), 1), "peak_per_direction_nominal": NVLINK_NOMINAL,
+            "frac_of_nvlink_nominal_per_pair": round(payload / len(pairs) / (ms * 1e6) / NVLINK_NOMINAL, 3),
+            "kernel_GBps_payload_max_rank": round(k_gbps, 1), "kernel_launches_per_xfer": int(kl // 5) if kl else 0,
             "bit_exact": bad == 0, "all_to_all": a2a}
 
 
