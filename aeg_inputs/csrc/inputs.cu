@@ -97,6 +97,14 @@ __global__ void gate(const volatile int* flag) {
   while (*flag == 0) __nanosleep(1000);
 }
 
+// GPU-wide nanosecond clock, comparable across processes sharing the GPU (cross-process timing of
+// the host-route hand-off, where CUDA events cannot be shared with timing enabled).
+__global__ void stamp(unsigned long long* out) {
+  unsigned long long t;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+  *out = t;
+}
+
 __global__ void spin(long long cycles) {
   const long long t0 = clock64();
   while (clock64() - t0 < cycles) {
@@ -238,11 +246,17 @@ int aegin_preload(void) {
   if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, consume_chunks);
   if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, gate);
   if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, spin);
+  if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, stamp);
   return int(e);
 }
 
 int aegin_gate(const void* pinned_flag, void* stream) {
   gate<<<1, 1, 0, static_cast<cudaStream_t>(stream)>>>(static_cast<const volatile int*>(pinned_flag));
+  return int(cudaGetLastError());
+}
+
+int aegin_stamp(void* dev_u64, void* stream) {
+  stamp<<<1, 1, 0, static_cast<cudaStream_t>(stream)>>>(static_cast<unsigned long long*>(dev_u64));
   return int(cudaGetLastError());
 }
 

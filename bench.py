@@ -848,6 +848,152 @@ def migrate_leg_dist(aeg, torch, dist, kernel, n_req=16):
             "bit_exact": bad == 0, "all_to_all": a2a}
 
 
+def _host_route_geometry(aeg, n_req):
+    import aeg_inputs as gi
+    sht = gi.KV_SHAPES["llama-2-13b"]
+    sh = aeg.KVShape.of(sht)
+    lens = gi.request_lengths(3, n_req, 512, 4096)
+    n = sum(-(-t // 16) for t in lens)
+    slab = GIB + 256 * MIB
+    nslab = -(-n // (slab // sh.block_bytes())) + 1
+    return sht, sh, n, slab, nslab
+
+
+def _dbg(*a):
+    if os.environ.get("AEG_DEBUG_ROUTE"):
+        print(f"[{os.getpid()} {time.time():.3f}]", *a, file=sys.stderr, flush=True)
+
+
+def _host_route_decode(conn, n_req):
+    """Decode instance D of the host-route leg (a separate process on the same GPU): imports the
+    prefill instance's node-shared CPU KV cache once, then per hand-off swaps the request in from
+    there (C->D, aeg_kv_swap_in_from) waiting only on P's per-layer IPC events, and stamps the GPU
+    clock when its last layer is ready."""
+    try:
+        import torch
+        import aeg_inputs as gi
+        from aeg_inputs import dev as D
+        import paper_conf_sosp_xiang0qyzyzl0025_b200 as aeg
+        sht, sh, n, slab, nslab = _host_route_geometry(aeg, n_req)
+        ctx = aeg.Context(0, aeg.default_config(device_kv_bytes=nslab * slab, host_kv_bytes=GIB, dev_slab_bytes=slab,
+                                                dev_slab_layout=aeg.BLOCK_MAJOR))
+        base, _ = ctx.pool_region(0)
+        _dbg("D: ctx up")
+        ctx.import_peer(0, conn.recv())
+        _dbg("D: peer imported")
+        t = torch.zeros(1, dtype=torch.int64, device="cuda")
+        s = torch.cuda.Stream()
+        D.stamp(t.data_ptr(), s.cuda_stream)   # load every kernel now: a module load later would wait
+        s.synchronize()                        # behind P's gate kernel
+        conn.send("ready")
+        keys = np.array([gi.kv_key(1, i // 4096, i % 4096, l) for i in range(n) for l in range(sh.num_layers)], np.uint64)
+        while True:
+            m = conn.recv()
+            if m == "bye":
+                break
+            hb, xblob = m
+            xo = ctx.xfer_import(0, xblob)
+            _dbg("D: events imported")
+            dc = ctx.kv_alloc(0, sht, n)
+            xi = ctx.kv_swap_in_from(sht, 0, np.array(hb, dtype=np.uint64), dc, after=xo)       # ③④⑤
+            _dbg("D: swap-in enqueued")
+            ctx.layer_ready(xi, -1, aeg.READY_WAIT_STREAM, s.cuda_stream)
+            D.stamp(t.data_ptr(), s.cuda_stream)
+            conn.send(ctx.xfer_export(xi))
+            _dbg("D: exported")
+            s.synchronize()
+            bad, _ = D.verify_chunks(base, chunk_offsets(ctx, 0, sht, dc), keys, sh.chunk_bytes(), gi.kv_seed(3))
+            ctx.xfer_release(xi)
+            ctx.xfer_release(xo)
+            ctx.kv_free(0, dc)
+            conn.send((int(t.item()), int(bad)))
+        ctx.shutdown()
+    except BaseException:
+        import traceback
+        conn.send(("error", traceback.format_exc()))
+
+
+def host_route_leg(aeg, torch, kernel, n_req=4, reps=4):
+    """NEXT-2, the paper's own P->C->D route (Fig. 10) measured: prefill instance
+    P (this process) swaps a hand-off of n_req Llama-2-13B requests out to its part of the node-shared
+    pinned CPU KV cache (P->C), decode instance D (another process, same GPU) swaps it in from there
+    (C->D) with per-layer IPC-event waits, so the two PCIe directions overlap layer by layer; P keeps
+    the CPU blocks in its move list until D's swap-in completes (aeg_kv_free_after).  Latency = GPU
+    clock from P's start to D's last layer ready (%globaltimer, shared by both processes)."""
+    import multiprocessing as mp
+    import aeg_inputs as gi
+    from aeg_inputs import dev as D
+    sht, sh, n, slab, nslab = _host_route_geometry(aeg, n_req)
+    a = aeg.Context(0, aeg.default_config(device_kv_bytes=nslab * slab, host_kv_bytes=nslab * slab,
+                                          dev_slab_bytes=slab, host_slab_bytes=slab, kernel=kernel,
+                                          flags=aeg.CFG_SHARED_HOST))
+    cm = mp.get_context("spawn")
+    parent, child = cm.Pipe()
+    p = cm.Process(target=_host_route_decode, args=(child, n_req))
+    p.start()
+    child.close()
+
+    def recv():
+        if not parent.poll(300):
+            raise RuntimeError("decode process did not answer")
+        m = parent.recv()
+        if isinstance(m, tuple) and len(m) == 2 and m[0] == "error":
+            raise RuntimeError("decode process failed:\n" + m[1])
+        return m
+
+    res = []
+    try:
+        abase, _ = a.pool_region(0)
+        src = a.kv_alloc(0, sht, n)
+        keys = [gi.kv_key(1, i // 4096, i % 4096, l) for i in range(n) for l in range(sh.num_layers)]
+        D.fill_chunks(abase, chunk_offsets(a, 0, sht, src), keys, sh.chunk_bytes(), gi.kv_seed(3))
+        D.sync()
+        parent.send(a.export_ipc())
+        if recv() != "ready":
+            raise RuntimeError("decode process handshake")
+        ts = torch.zeros(2, dtype=torch.int64, device="cuda")
+        s, s2 = torch.cuda.Stream(), torch.cuda.Stream()
+        gate = D.Gate()
+        for _ in range(reps + 1):
+            hc = a.kv_alloc(1, sht, n)
+            _dbg("P: rep")
+            gate.close_on(s.cuda_stream)          # everything is enqueued on both sides before it starts
+            D.stamp(ts.data_ptr(), s.cuda_stream)
+            a.stream_fence(s.cuda_stream)
+            xo = a.kv_swap_out(sht, src, hc)                                                       # ①②
+            parent.send(([int(b) for b in hc], a.xfer_export(xo)))
+            _dbg("P: swap-out enqueued + sent")
+            xd = a.xfer_import(1, recv())
+            _dbg("P: D's events imported")
+            a.layer_ready(xo, -1, aeg.READY_WAIT_STREAM, s2.cuda_stream)
+            D.stamp(ts.data_ptr() + 8, s2.cuda_stream)
+            a.kv_free_after(1, hc, xd)            # the CPU blocks stay in P's move list until D is done
+            gate.open()
+            _dbg("P: gate open")
+            t_end, bad = recv()
+            _dbg("P: rep done")
+            torch.cuda.synchronize()
+            t0, t_out = (int(x) for x in ts.tolist())
+            a.xfer_release(xo)
+            a.xfer_release(xd)
+            res.append((t_out - t0, t_end - t0, bad))
+        parent.send("bye")
+    finally:
+        p.join(timeout=60)
+        if p.is_alive():
+            p.kill()
+        a.shutdown()
+    res = res[1:]
+    b = n * sh.block_bytes()
+    out_ns = statistics.median(r[0] for r in res)
+    e2e_ns = statistics.median(r[1] for r in res)
+    return {"workload": f"configs[2] Llama-2-13B hand-off of {n_req} requests ({n} blocks, {b / GIB:.2f} GiB) through "
+                        "the node-shared pinned CPU cache, P and D in two processes on one GPU",
+            "p_to_c_ms": round(out_ns / 1e6, 2), "p_to_c_GBps": round(b / out_ns, 1),
+            "p_to_d_ms": round(e2e_ns / 1e6, 2), "p_to_d_GBps": round(b / e2e_ns, 1),
+            "bit_exact": all(r[2] == 0 for r in res), "reps": len(res)}
+
+
 def sparse_model_cache(name, m, tp_rank, tp_size, seed, threads=16, min_sparse=MIB):
     """Host Model Cache of a whole model (pageable) laid out as model_caches()
     does, but only TP rank `tp_rank`'s shard bytes are materialised: the rest of the anonymous
@@ -1328,11 +1474,12 @@ def run_ours(args):
         else:
             c5 = {"skipped": "configs[4] is the 8-GPU TP=4 layout (one rank pair on 1 GPU); not defined for N=%d" % world}
         small = None if world > 1 else leg("small_chunk", lambda: small_chunk_leg(aeg, torch, kernel))
+        route = None if world > 1 else leg("host_route", lambda: host_route_leg(aeg, torch, kernel))
         alloc = leg("allocator", lambda: allocator_leg(aeg)) if rank == 0 else None
         cpu = None if args.no_cpu or rank != 0 else leg("cpu_baseline", cpu_baseline)
         out.update({"e2e": e2e, "verify": ver, "one_direction": one_dir, "pcie_memcpy_GBps": {k: round(v, 1) for k, v in pc.items()},
                     "switch": sw, "migrate": mig, "per_layer_overlap": ovl, "c5": c5, "allocator": alloc,
-                    "per_chunk_memcpy_baseline": base, "small_chunk": small,
+                    "per_chunk_memcpy_baseline": base, "small_chunk": small, "host_route": route,
                     "cpu_baseline": cpu})
         if not ver.get("ok"):
             log("VERIFICATION FAILED", ver)

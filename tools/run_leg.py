@@ -1,5 +1,5 @@
 """Run one bench.py side leg alone on cuda:0 and print its JSON (development / profiling helper).
-    python tools/run_leg.py c5|migrate|overlap [kernel]"""
+    python tools/run_leg.py c5|migrate|overlap|small_chunk|switch|host_route [auto|lsu|bulk]"""
 import json
 import os
 import sys
@@ -11,23 +11,34 @@ import bench  # noqa: E402
 import paper_conf_sosp_xiang0qyzyzl0025_b200 as aeg  # noqa: E402
 from paper_conf_sosp_xiang0qyzyzl0025_b200 import build  # noqa: E402
 
-build.build()
-leg = sys.argv[1]
-kernel = {"auto": aeg.KERNEL_AUTO, "lsu": aeg.KERNEL_LSU, "bulk": aeg.KERNEL_BULK}[sys.argv[2] if len(sys.argv) > 2 else "auto"]
-fn = {"c5": lambda: bench.c5_leg(aeg, torch, kernel), "migrate": lambda: bench.migrate_leg(aeg, torch, kernel),
-      "overlap": lambda: bench.overlap_leg(aeg, torch, kernel),
-      "small_chunk": lambda: bench.small_chunk_leg(aeg, torch, kernel), "switch": lambda: switch_cmp()}[leg]
 
-
-def switch_cmp():
+def switch_cmp(kernel):
     """configs[3] switch with A's KV-out concurrent with B's load vs after it, per weight mode."""
     descs, caches = bench.model_caches(["qwen-1.8b", "llama-7b", "yi-9b"])
     out = {}
     for mode in ("staged", "prefetch", "direct"):
         for kv_out in ("concurrent", "after"):
             r = bench.switch_leg(aeg, torch, 12, kernel, descs, mode, caches if mode == "direct" else None, kv_out)
-            out[f"{mode}/{kv_out}"] = {k: (v["last_layer_ms_p50"], v["first_layer_ms_p50"]) for k, v in r["per_model"].items()}
-            out[f"{mode}/{kv_out}"]["landing"] = r["landing_ms_one_switch"]
-            print(json.dumps({f"{mode}/{kv_out}": out[f"{mode}/{kv_out}"]}), flush=True)
+            key = f"{mode}/{kv_out}"
+            out[key] = {k: (v["last_layer_ms_p50"], v["first_layer_ms_p50"]) for k, v in r["per_model"].items()}
+            out[key]["landing"] = r["landing_ms_one_switch"]
+            print(json.dumps({key: out[key]}), flush=True)
     return out
-print(json.dumps(fn()), flush=True)
+
+
+def main():
+    build.build()
+    leg = sys.argv[1]
+    kernel = {"auto": aeg.KERNEL_AUTO, "lsu": aeg.KERNEL_LSU, "bulk": aeg.KERNEL_BULK}[
+        sys.argv[2] if len(sys.argv) > 2 else "auto"]
+    fn = {"c5": lambda: bench.c5_leg(aeg, torch, kernel),
+          "migrate": lambda: bench.migrate_leg(aeg, torch, kernel),
+          "overlap": lambda: bench.overlap_leg(aeg, torch, kernel),
+          "small_chunk": lambda: bench.small_chunk_leg(aeg, torch, kernel),
+          "switch": lambda: switch_cmp(kernel),
+          "host_route": lambda: bench.host_route_leg(aeg, torch, kernel)}[leg]
+    print(json.dumps(fn()), flush=True)
+
+
+if __name__ == "__main__":
+    main()
