@@ -262,3 +262,11 @@ def test_big_pool_alloc_is_fast():
     got = c.kv_alloc(aeg.POOL_DEVICE, sh, 1024)
     assert len(set(got.tolist())) == 1024
     c.shutdown()
+
+
+def test_bench_allocator_leg_runs_on_a_host_only_context():
+    """bench.py's H1 control-overhead leg needs no GPU (host-only context, C2 geometry, aged pool)."""
+    import bench
+    r = bench.allocator_leg(aeg, reps=2)
+    assert r["per_request_alloc_us_p50"] > 0 and r["batch_alloc_ns_per_block"] > 0
+    assert r["batch_free_us"] > 0 and "3970" in r["workload"]
