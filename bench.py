@@ -757,6 +757,34 @@ def migrate_leg(aeg, torch, kernel, n_req=16, src_layout=None, dst_layout=None):
             "per_chunk_memcpy_calls": int(len(offs))}
 
 
+def _nccl_sendrecv(torch, dist, pairs, nbytes, reps=4):
+    """NCCL point-to-point of one hand-off's payload as ONE contiguous buffer per pair (no block
+    tables, no gather/scatter: an upper bound for an NCCL-based hand-off).  Max-over-ranks device
+    time of the median rep."""
+    td = dist.td
+    rank = dist.rank
+    peer = {a_: b_ for a_, b_ in pairs}
+    peer.update({b_: a_ for a_, b_ in pairs})
+    if rank not in peer:
+        return None
+    buf = torch.empty(nbytes, dtype=torch.uint8, device="cuda")
+    ts = []
+    for _ in range(reps + 1):
+        dist.barrier()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record()
+        if any(a_ == rank for a_, _ in pairs):
+            td.send(buf, peer[rank])
+        else:
+            td.recv(buf, peer[rank])
+        e1.record()
+        e1.synchronize()
+        ts.append(dist.max(e0.elapsed_time(e1)))
+    del buf
+    ms = statistics.median(ts[1:])
+    return {"ms": round(ms, 3), "GBps_per_pair": round(nbytes / (ms * 1e6), 1)}
+
+
 def migrate_leg_dist(aeg, torch, dist, kernel, n_req=16):
     """configs[2] across GPUs: prefill rank i hands n_req Llama-2-13B-shaped requests to decode rank
     i + N/2 over NVLink/NVSwitch (fused gather -> remote 16-byte stores), per-layer IPC events.
@@ -838,9 +866,13 @@ def migrate_leg_dist(aeg, torch, dist, kernel, n_req=16):
         a2a = {"rounds": h, "ms_total": round(sum(t_rounds), 3),
                "GBps_aggregate": round(h * len(pairs) * n * sh.block_bytes() / (sum(t_rounds) * 1e6), 1)}
     ctx.shutdown()
+    nccl = None
+    if dist.backend == "nccl":   # comparison baseline (not the product): NCCL send/recv of the same
+        nccl = _nccl_sendrecv(torch, dist, pairs, n * sh.block_bytes())   # payload, contiguous
     ms = statistics.median(times)
     payload = len(pairs) * n * sh.block_bytes()
     return {"workload": f"configs[2] Llama-2-13B hand-off, {n_req} requests per pair, pairs {pairs}",
+            "nccl_sendrecv_contiguous_baseline": nccl,
             "payload_bytes": payload, "ms": round(ms, 3), "GBps_aggregate": round(payload / (ms * 1e6), 1),
             "GBps_per_pair": round(payload / len(pairs) / (ms * 1e6), 1), "peak_per_direction_nominal": NVLINK_NOMINAL,
             "frac_of_nvlink_nominal_per_pair": round(payload / len(pairs) / (ms * 1e6) / NVLINK_NOMINAL, 3),
