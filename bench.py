@@ -765,17 +765,15 @@ def _nccl_sendrecv(torch, dist, pairs, nbytes, reps=4):
     rank = dist.rank
     peer = {a_: b_ for a_, b_ in pairs}
     peer.update({b_: a_ for a_, b_ in pairs})
-    if rank not in peer:
-        return None
-    buf = torch.empty(nbytes, dtype=torch.uint8, device="cuda")
+    buf = torch.empty(nbytes, dtype=torch.uint8, device="cuda") if rank in peer else None
     ts = []
-    for _ in range(reps + 1):
+    for _ in range(reps + 1):   # every rank takes part in the barrier / max, paired or not
         dist.barrier()
         e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         e0.record()
-        if any(a_ == rank for a_, _ in pairs):
+        if buf is not None and any(a_ == rank for a_, _ in pairs):
             td.send(buf, peer[rank])
-        else:
+        elif buf is not None:
             td.recv(buf, peer[rank])
         e1.record()
         e1.synchronize()
