@@ -717,20 +717,31 @@ def migrate_leg(aeg, torch, kernel, n_req=16, src_layout=None, dst_layout=None):
     keys = [gi.kv_key(1, i // 4096, i % 4096, l) for i in range(n) for l in range(sh.num_layers)]
     D.fill_chunks(abase, offs, keys, sh.chunk_bytes(), seed)
     a.import_peer(1, b.export_ipc())
-    times = []
-    for it in range(6):
-        a.kernel_stats_reset()
-        s = torch.cuda.Stream()
-        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-        e0.record(s)
-        a.stream_fence(s.cuda_stream)
-        x = a.kv_migrate(sht, sc, 1, dc)
-        a.layer_ready(x, -1, aeg.READY_WAIT_STREAM, s.cuda_stream)
-        e1.record(s)
-        e1.synchronize()
-        a.xfer_release(x)
-        if it >= 2:
-            times.append(e0.elapsed_time(e1))
+
+    def timed(reps):
+        out = []
+        for it in range(reps + 2):
+            a.kernel_stats_reset()
+            s = torch.cuda.Stream()
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record(s)
+            a.stream_fence(s.cuda_stream)
+            x = a.kv_migrate(sht, sc, 1, dc)
+            a.layer_ready(x, -1, aeg.READY_WAIT_STREAM, s.cuda_stream)
+            e1.record(s)
+            e1.synchronize()
+            a.xfer_release(x)
+            if it >= 2:
+                out.append(e0.elapsed_time(e1))
+        return out
+
+    # SM budget of the hand-off (aeg_set_migrate_ctas): CTAs of 256 threads, ~one per SM up to 148
+    sweep = {}
+    for ctas in (8, 16, 32, 64, 148):
+        a.set_migrate_ctas(ctas)
+        sweep[ctas] = round(n * sh.block_bytes() / (min(timed(2)) * 1e6), 1)
+    a.set_migrate_ctas(0)
+    times = timed(4)
     nl, nbytes, kms = a.kernel_stats(aeg.K_MIGRATE)
     doffs = chunk_offsets(b, 0, sht, dc)
     bad, _ = D.verify_chunks(bbase, doffs, keys, sh.chunk_bytes(), seed)
@@ -753,6 +764,7 @@ def migrate_leg(aeg, torch, kernel, n_req=16, src_layout=None, dst_layout=None):
             "payload_bytes": payload, "ms": round(ms, 3), "GBps_payload": round(payload / (ms * 1e6), 1),
             "hbm_GBps": round(2 * payload / (ms * 1e6), 1), "kernel_launches_per_xfer": nl,
             "kernel_ms_per_xfer": round(kms, 3), "bit_exact": bad == 0,
+            "GBps_payload_by_ctas": sweep,
             "per_chunk_memcpy_baseline_GBps_payload": round(payload / (min(bt) * 1e6), 1),
             "per_chunk_memcpy_calls": int(len(offs))}
 
@@ -849,6 +861,11 @@ def migrate_leg_dist(aeg, torch, dist, kernel, n_req=16):
     times = [hand_off(pairs) for _ in range(5)][1:]
     kl, kb, kms = ctx.kernel_stats(aeg.K_MIGRATE)   # prefill ranks: 5 rounds of migrate launches
     k_gbps = dist.max(kb / 2 / (kms * 1e6) if kms > 0 else 0.0)   # payload bytes over the link
+    sweep = {}   # SM budget of the hand-off: how many SMs saturate the link
+    for ctas in (8, 16, 32, 64, 148):
+        ctx.set_migrate_ctas(ctas)
+        sweep[ctas] = round(len(pairs) * n * sh.block_bytes() / (min(hand_off(pairs) for _ in range(2)) * 1e6), 1)
+    ctx.set_migrate_ctas(0)
     bad = 0
     if not prefill:
         sender = [s_ for s_, d in pairs if d == rank][0]
@@ -875,6 +892,7 @@ def migrate_leg_dist(aeg, torch, dist, kernel, n_req=16):
             "GBps_per_pair": round(payload / len(pairs) / (ms * 1e6), 1), "peak_per_direction_nominal": NVLINK_NOMINAL,
             "frac_of_nvlink_nominal_per_pair": round(payload / len(pairs) / (ms * 1e6) / NVLINK_NOMINAL, 3),
             "kernel_GBps_payload_max_rank": round(k_gbps, 1), "kernel_launches_per_xfer": int(kl // 5) if kl else 0,
+            "GBps_aggregate_by_ctas": sweep,
             "bit_exact": bad == 0, "all_to_all": a2a}
 
 

@@ -321,6 +321,12 @@ int aeg_import_peer(aeg_ctx ctx, int32_t peer, const void* buf, uint64_t len);
 int aeg_xfer_export(aeg_ctx ctx, aeg_xfer x, void* buf, uint64_t* len);
 int aeg_xfer_import(aeg_ctx ctx, int32_t peer, const void* buf, uint64_t len, aeg_xfer* out);
 
+/* SM budget of later aeg_kv_migrate launches (aeg_config.migrate_ctas at run time): ctas > 0 caps
+ * the migrate kernel's grid at `ctas` CTAs of 256 threads (the block scheduler spreads them one per
+ * SM first, so ctas <= 148 ~ that many SMs), leaving the rest of the GPU to the decode instance's
+ * compute; 0 = a full wave.  AEG_ERR_INVALID if ctas < 0.  Transfers already enqueued keep theirs. */
+int aeg_set_migrate_ctas(aeg_ctx ctx, int32_t ctas);
+
 /* ---- instrumentation ---------------------------------------------------------------------- */
 
 /* Kernel counters since the last reset (needs AEG_CFG_TIMING for ms): kind 0 gather, 1 scatter,

@@ -120,6 +120,7 @@ _SIGS = {
     "aeg_xfer_import": [P, I32, P, U64, PU64],
     "aeg_kernel_stats": [P, I32, PU64, PU64, C.POINTER(C.c_double)],
     "aeg_kernel_stats_reset": [P],
+    "aeg_set_migrate_ctas": [P, C.c_int32],
     "aeg_trace_enable": [P, C.c_int],
     "aeg_trace_read": [P, C.c_char_p, PU64],
     "aeg_debug_xfer_begin": [P, I32, PU64, I32, PU64],
@@ -357,6 +358,9 @@ class Context:
         n, b, ms = C.c_uint64(), C.c_uint64(), C.c_double()
         _chk(lib().aeg_kernel_stats(self.h, int(kind), C.byref(n), C.byref(b), C.byref(ms)))
         return n.value, b.value, ms.value
+
+    def set_migrate_ctas(self, ctas: int):
+        _chk(lib().aeg_set_migrate_ctas(self.h, int(ctas)))
 
     def kernel_stats_reset(self):
         _chk(lib().aeg_kernel_stats_reset(self.h))

@@ -629,6 +629,16 @@ int aeg_kernel_stats(aeg_ctx ctx, int32_t kind, uint64_t* launches, uint64_t* by
   });
 }
 
+int aeg_set_migrate_ctas(aeg_ctx ctx, int32_t ctas) {
+  return guarded([&] {
+    Ctx& c = C(ctx);
+    AEG_REQUIRE(ctas >= 0, AEG_ERR_INVALID, "ctas must be >= 0");
+    std::lock_guard<std::mutex> g(c.mu);
+    c.cfg.migrate_ctas = ctas;
+    return AEG_OK;
+  });
+}
+
 int aeg_kernel_stats_reset(aeg_ctx ctx) {
   return guarded([&] {
     Ctx& c = C(ctx);

@@ -48,6 +48,29 @@ def test_local_migrate(kernel):
         ctx.shutdown()
 
 
+@pytest.mark.parametrize("ctas", [1, 3])
+def test_local_migrate_under_an_sm_budget(ctas):
+    """aeg_set_migrate_ctas: a grid of 1 or 3 CTAs strides over every (block, layer) piece."""
+    require_gpu()
+    ctx, dev = make(aeg.LAYER_MAJOR, kernel=aeg.KERNEL_AUTO)
+    try:
+        with pytest.raises(aeg.AegError):
+            ctx.set_migrate_ctas(-1)
+        ctx.set_migrate_ctas(ctas)
+        dev.poison(gi.TAG_NEVER)
+        img = dev.poison_img(gi.TAG_NEVER)
+        sc, so = dev.alloc(SH, 29)
+        fill_blocks(dev, img, SH, so, [(0, j) for j in range(29)])
+        dc, do = dev.alloc(SH, 29)
+        poison_blocks(dev, img, SH, do)
+        x = ctx.kv_migrate(SH.as_tuple(), sc, -1, dc)
+        exp = OK.migrate(img, dev.geom, img, dev.geom, SH, so, do)
+        ctx.layer_ready(x, -1, aeg.READY_BLOCK)
+        assert first_diff(dev.read(), exp) is None
+    finally:
+        ctx.shutdown()
+
+
 def test_same_process_peer_migrate_and_imported_events():
     require_gpu()
     a, A = make(aeg.LAYER_MAJOR, slab=MIB)
