@@ -175,15 +175,17 @@ static void host_dmas(const SlabPool& hp, char* hbase, const Shape& sh, const st
 // (plain st.global to peer addresses) unless BULK is requested explicitly.
 #define ipc_events(flags) (((flags) & AEG_IPC_EVENTS) || (cfg.flags & AEG_CFG_SHARED_HOST))
 
-// AUTO by chunk size, from tools/launch_probe.cu (profiles/r01/launch_probe2.txt, TB/s body):
+// AUTO by chunk size, from tools/launch_probe.cu (profiles/r01/launch_probe2.txt, TB/s body) and
+// tools/threshold_probe.cu (profiles/r01/threshold_probe.txt, ~1 GiB launches, gather / scatter):
 //   2 KiB chunks: WARP 5.1, LSU 1.7, BULK 0.8     8 KiB: LSU 4.8-5.4, WARP 1.5-4.3, BULK 2.7-2.9
-//   256 KiB: BULK 6.1-6.3, LSU 5.8-6.0
+//   16 KiB: LSU 6.0 / 5.9, BULK 5.1 / 5.2         32 KiB: BULK 6.2 / 6.6, LSU 5.8 / 5.8
+//   64-512 KiB: BULK 6.1-6.5, LSU 5.9
 static int impl_of(const aeg_config& cfg, uint64_t chunk) {
   if (cfg.kernel == AEG_KERNEL_LSU) return IMPL_LSU;
   if (cfg.kernel == AEG_KERNEL_BULK) return IMPL_BULK;
   if (cfg.kernel == AEG_KERNEL_WARP) return IMPL_WARP;
   if (chunk <= (4u << 10)) return IMPL_WARP;
-  return chunk < (64u << 10) ? IMPL_LSU : IMPL_BULK;
+  return chunk < (32u << 10) ? IMPL_LSU : IMPL_BULK;
 }
 
 // ----------------------------------------------------------------------------- swap-out H3
