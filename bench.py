@@ -495,8 +495,45 @@ def pcie_calibration(torch):
             e1.record()
         e1.synchronize()
         out[name] = 3 * GIB / (e0.elapsed_time(e1) * 1e6)
-    del h, d
+    # both directions at once (the ceiling of the round-trip `value`): 3 x 1 GiB each way
+    h2 = torch.empty(GIB, dtype=torch.uint8, pin_memory=True)
+    d2 = torch.empty(GIB, dtype=torch.uint8, device="cuda")
+    s2 = torch.cuda.Stream()
+    torch.cuda.synchronize()
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    e0.record(s)
+    s2.wait_event(e0)
+    for _ in range(3):
+        with torch.cuda.stream(s):
+            d.copy_(h, non_blocking=True)
+        with torch.cuda.stream(s2):
+            h2.copy_(d2, non_blocking=True)
+    s.wait_stream(s2)
+    e1.record(s)
+    e1.synchronize()
+    out["bidir_total"] = 6 * GIB / (e0.elapsed_time(e1) * 1e6)
+    del h, d, h2, d2
     return out
+
+
+def host_facts():
+    """The box the numbers were taken on: CPU count / model, memory, NUMA nodes, the
+    GPU's NUMA node."""
+    import platform
+    f = {"cpus": os.cpu_count(), "machine": platform.machine()}
+    try:
+        for line in open("/proc/cpuinfo"):
+            if line.startswith("model name"):
+                f["cpu_model"] = line.split(":", 1)[1].strip()
+                break
+        for line in open("/proc/meminfo"):
+            if line.startswith("MemTotal"):
+                f["mem_gib"] = round(int(line.split()[1]) / 2**20, 1)
+                break
+        f["numa_nodes"] = len([d for d in os.listdir("/sys/devices/system/node") if d.startswith("node")])
+    except OSError:
+        pass
+    return f
 
 
 def model_caches(names):
@@ -1528,6 +1565,7 @@ def run_ours(args):
         out.update({"e2e": e2e, "verify": ver, "one_direction": one_dir, "pcie_memcpy_GBps": {k: round(v, 1) for k, v in pc.items()},
                     "switch": sw, "migrate": mig, "per_layer_overlap": ovl, "c5": c5, "allocator": alloc,
                     "per_chunk_memcpy_baseline": base, "small_chunk": small, "host_route": route,
+                    "host": host_facts(),
                     "cpu_baseline": cpu})
         if not ver.get("ok"):
             log("VERIFICATION FAILED", ver)
@@ -1560,6 +1598,10 @@ def run_ours(args):
             "consumer_launches": args.steps * sb.L,
         }
         res.update(out)
+        pm = out.get("pcie_memcpy_GBps") or {}
+        if pm.get("bidir_total"):   # the round trip against this box's own duplex copy-engine ceiling
+            res["pcie"]["measured_bidir_memcpy_GBps"] = round(pm["bidir_total"], 1)
+            res["pcie"]["frac_of_measured_bidir"] = round(value / pm["bidir_total"], 3)
         od = out.get("one_direction")
         if od and "error" not in od:   # each direction alone against PCIe Gen5 x16 nominal 64 GB/s (target >= 0.80)
             res["pcie"]["swap_out_alone_GBps"] = od["swap_out"]["GBps"]
