@@ -71,6 +71,7 @@ def parse():
     p.add_argument("--switches", type=int, default=30)
     p.add_argument("--slot-mib", type=int, default=0, help="staging slot size (0 = library default)")
     p.add_argument("--slots", type=int, default=0)
+    p.add_argument("--dma-piece-mib", type=int, default=0, help="swap-out D2H piece (0 = library default)")
     p.add_argument("--profile", action="store_true", help="short run for ncu (no side legs)")
     return p.parse_args()
 
@@ -226,7 +227,7 @@ class SwapBench:
     tests/oracle_swapbench.py (test infrastructure)."""
 
     def __init__(self, aeg, sh, n_req, kernel, extra_host_slabs=8, weight_bytes=0, seed_cfg=2, slot_mib=0, slots=0,
-                 churn_slabs=12):
+                 churn_slabs=12, dma_piece_mib=0):
         import aeg_inputs as gi
         self.aeg, self.gi = aeg, gi
         self.sht = sh
@@ -248,6 +249,8 @@ class SwapBench:
             cfg.staging_slot_bytes = slot_mib * MIB
         if slots:
             cfg.staging_slots = slots
+        if dma_piece_mib:
+            cfg.dma_piece_mib = dma_piece_mib
         self.cfg = cfg
         t0 = time.time()
         import torch
@@ -336,21 +339,43 @@ class SwapBench:
         t = off0[None, :] + np.arange(self.L, dtype=np.uint64)[:, None] * np.uint64(stride)
         return torch.from_numpy(t.astype(np.int64)).cuda()
 
-    def step(self, torch, cons, with_consumer=True, record=True, keep_host_offsets=False):
-        """One timed step, library calls only (plus the synthetic consumer)."""
+    def step(self, torch, cons, with_consumer=True, record=True, keep_host_offsets=False, first_layer=None):
+        """One timed step, library calls only (plus the synthetic consumer).  first_layer: a list
+        that receives (start, layer-0-ready, last-layer-ready) events on the consumer stream."""
         aeg = self.aeg
         from aeg_inputs import dev as D
+        if first_layer is not None:
+            ev = [torch.cuda.Event(enable_timing=True) for _ in range(3)]
+            ev[0].record(cons)
+            first_layer.extend(ev)
         hc = self.ctx.kv_alloc(aeg.POOL_HOST, self.sht, self.n)
         if keep_host_offsets:   # the host blocks are freed (and their slabs may be reclaimed) by the swap-in
             self.host_offs = self.chunk_offsets(1, hc)
         nd = self.ctx.kv_alloc(aeg.POOL_DEVICE, self.sht, self.n)
+        # the consumer's block table is uploaded before the transfers are queued: a pageable H2D
+        # copy queued behind the swap-in's DMAs would wait for all of them (one copy engine serves
+        # H2D streams FIFO, profiles/r01/ce_probe.txt) and hold the host back from enqueueing the
+        # per-layer waits
+        tab = self.consumer_tables(torch, nd) if with_consumer else None
         self.ctx.stream_fence(cons.cuda_stream)
+        t0 = time.perf_counter()
         x = self.ctx.kv_swap_out(self.sht, self.src_c, hc, flags=aeg.FREE_SRC)
+        t1 = time.perf_counter()
         y = self.ctx.kv_swap_in(self.sht, hc, nd, flags=aeg.FREE_SRC)
+        t2 = time.perf_counter()
+        if first_layer is not None:   # diagnostics: host enqueue time of each call, swap-out layer 0 landed
+            self.enqueue_ms = ((t1 - t0) * 1e3, (t2 - t1) * 1e3)
+            if not hasattr(self, "diag_stream"):
+                self.diag_stream = torch.cuda.Stream()
+            self.ctx.layer_ready(x, 0, aeg.READY_WAIT_STREAM, self.diag_stream.cuda_stream)
+            ex = torch.cuda.Event(enable_timing=True)
+            ex.record(self.diag_stream)
+            first_layer.append(ex)
         if with_consumer:
-            tab = self.consumer_tables(torch, nd)
             for l in range(self.L):
                 self.ctx.layer_ready(y, l, aeg.READY_WAIT_STREAM, cons.cuda_stream)
+                if first_layer is not None and l in (0, self.L - 1):
+                    first_layer[1 if l == 0 else 2].record(cons)
                 D.consume(self.dbase, tab[l].data_ptr(), self.n, self.Cl, self.sink.data_ptr(), cons.cuda_stream)
         else:
             self.ctx.layer_ready(y, -1, aeg.READY_WAIT_STREAM, cons.cuda_stream)
@@ -399,7 +424,8 @@ class SwapBench:
 def chunk_memcpy_baseline(aeg, torch, ctx, sht, src_blocks, reps=2):
     """The per-block memcpy the paper's swap amounts to for paged KV ("memcpy(async)"
     Fig. 10; vLLM-style swap_blocks): one cudaMemcpyAsync per (block, layer) chunk, device blocks ->
-    host blocks, then host -> fresh device blocks, on one stream (copy engines only).  Same blocks and
+    host blocks, then host -> fresh device blocks, on one stream (copy engines only); and the same
+    chunks through the batched-memcpy API (cudaMemcpyBatchAsync, `batch_api_*`).  Same blocks and
     placement as the library's swap; timed with CUDA events.  Returns GB/s per direction."""
     from aeg_inputs import dev as D
     sh = aeg.KVShape.of(sht)
@@ -411,16 +437,17 @@ def chunk_memcpy_baseline(aeg, torch, ctx, sht, src_blocks, reps=2):
     so, ho, no = (chunk_offsets(ctx, p, sht, b) for p, b in ((0, src_blocks), (1, hc), (0, nd)))
     s = torch.cuda.Stream()
     out = {}
-    for name, args in (("d2h", (hbase, ho, dbase, so)), ("h2d", (dbase, no, hbase, ho))):
-        ts = []
-        for _ in range(reps):
-            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-            e0.record(s)
-            D.copy_chunks(*args, sh.chunk_bytes(), s.cuda_stream)
-            e1.record(s)
-            e1.synchronize()
-            ts.append(e0.elapsed_time(e1))
-        out[name + "_GBps"] = round(n * sh.block_bytes() / (min(ts) * 1e6), 2)
+    for fn, pre in ((D.copy_chunks, ""), (D.copy_chunks_batch, "batch_api_")):
+        for name, args in (("d2h", (hbase, ho, dbase, so)), ("h2d", (dbase, no, hbase, ho))):
+            ts = []
+            for _ in range(reps):
+                e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                e0.record(s)
+                fn(*args, sh.chunk_bytes(), s.cuda_stream)
+                e1.record(s)
+                e1.synchronize()
+                ts.append(e0.elapsed_time(e1))
+            out[pre + name + "_GBps"] = round(n * sh.block_bytes() / (min(ts) * 1e6), 2)
     out["memcpy_calls_per_direction"] = int(so.size)
     out["chunk_bytes"] = sh.chunk_bytes()
     ctx.kv_free(aeg.POOL_HOST, hc)
@@ -1464,6 +1491,7 @@ def run_ours(args):
         while n_req > 4 and sum(c2_requests(n_req)[1]) * 8 * MIB * 1.3 > per_rank:
             n_req //= 2
     sb = SwapBench(aeg, QWEN7B, n_req, kernel, slot_mib=args.slot_mib, slots=args.slots,
+                   dma_piece_mib=args.dma_piece_mib,
                    churn_slabs=args.churn_slabs).setup()
     sb.sink = torch.zeros(1, dtype=torch.int64, device="cuda")
     cons = torch.cuda.Stream()
@@ -1505,18 +1533,26 @@ def run_ours(args):
         # e2e: the same step through the public Python API, wall clock, after a host sync each step
         e2e = None
         if not args.no_e2e:
-            ts = []
+            ts, fl = [], []
             for _ in range(max(3, args.steps // 2)):
                 torch.cuda.synchronize()
                 t0 = time.perf_counter()
-                sb.step(torch, cons)
+                ev = []
+                sb.step(torch, cons, first_layer=ev)
                 cons.synchronize()
                 ts.append(time.perf_counter() - t0)
+                fl.append((ev[0].elapsed_time(ev[1]), ev[0].elapsed_time(ev[2]), ev[0].elapsed_time(ev[3]))
+                          + sb.enqueue_ms)
             e2e_t = dist.max(statistics.median(ts))   # the job's step ends when the slowest rank's does
             e2e = {"value": round(dist.sum(bytes_step) / e2e_t / 1e9, 2), "unit": "GB/s",
                    "h2d_bytes_per_step": int(bytes_step // 2 + 2 * sb.n * 8),
                    "d2h_bytes_per_step": int(bytes_step // 2),
-                   "how": "wall clock around the Python-API calls of one step incl. host sync"}
+                   "how": "wall clock around the Python-API calls of one step incl. host sync",
+                   "round_trip_layer0_ready_ms_p50": round(statistics.median(f[0] for f in fl), 2),
+                   "round_trip_last_layer_ready_ms_p50": round(statistics.median(f[1] for f in fl), 2),
+                   "swap_out_layer0_landed_ms_p50": round(statistics.median(f[2] for f in fl), 2),
+                   "enqueue_ms_p50": {"swap_out": round(statistics.median(f[3] for f in fl), 2),
+                                      "swap_in": round(statistics.median(f[4] for f in fl), 2)}}
         def leg(name, fn):
             """A side leg that fails reports its error in the line instead of losing the whole line."""
             try:
@@ -1583,6 +1619,7 @@ def run_ours(args):
                        "bytes_per_direction": sb.n * sb.sh.block_bytes(), "slab": "1 GiB layer-major",
                        "placement": "device pool aged by seeded churn", "l2": "inputs larger than L2 (32 GiB/step)",
                        "kernel": args.kernel, "staging_slot_mib": sb.cfg.staging_slot_bytes >> 20,
+                       "dma_piece_mib": sb.cfg.dma_piece_mib,
                        "staging_slots": sb.cfg.staging_slots, "parallelism": f"replicas x{world}"},
             "roofline": {"bound": "hbm", "kernel": "gather (swap-out, H2)", "achieved": round(g_ach, 1),
                          "peak": hbm, "peak_source": hbm_src, "unit": "GB/s",

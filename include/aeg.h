@@ -115,7 +115,10 @@ typedef struct {
   uint32_t flags;               /* AEG_CFG_*                                                  */
   int32_t numa_node;            /* pinned host memory placement: 0 = the GPU's NUMA node (from
                                    sysfs; unbound if unknown), n > 0 = node n-1, -1 = no binding */
-  uint32_t reserved[6];
+  uint32_t dma_piece_mib;       /* swap-out D2H piece (MiB) for sub-layer rule-❷ waits of a
+                                   chained swap-in; 0 = 128, >= 4096 = one piece
+                                   per segment (per-layer events only)                          */
+  uint32_t reserved[5];
 } aeg_config;
 
 /* One checkpoint tensor in the (pageable or registered) host Model Cache, row-major

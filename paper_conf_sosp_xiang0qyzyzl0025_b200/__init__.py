@@ -61,7 +61,8 @@ class Config(C.Structure):
                 ("staging_slot_bytes", C.c_uint64), ("table_arena_bytes", C.c_uint64),
                 ("dev_slab_layout", C.c_int32), ("host_slab_layout", C.c_int32), ("staging_slots", C.c_int32),
                 ("host_threads", C.c_int32), ("kernel", C.c_int32), ("migrate_ctas", C.c_int32),
-                ("flags", C.c_uint32), ("numa_node", C.c_int32), ("reserved", C.c_uint32 * 6)]
+                ("flags", C.c_uint32), ("numa_node", C.c_int32), ("dma_piece_mib", C.c_uint32),
+                ("reserved", C.c_uint32 * 5)]
 
 
 class WeightDesc(C.Structure):

@@ -104,6 +104,7 @@ int aeg_config_default(aeg_config* cfg) {
     cfg->dev_slab_layout = AEG_LAYER_MAJOR;
     cfg->host_slab_layout = AEG_LAYER_MAJOR;
     cfg->kernel = AEG_KERNEL_AUTO;
+    cfg->dma_piece_mib = 128;
     return AEG_OK;
   });
 }
@@ -122,6 +123,7 @@ int aeg_init(int device, const aeg_config* cfg, aeg_ctx* out) {
     if (!c.staging_slots) c.staging_slots = d.staging_slots;
     if (!c.table_arena_bytes) c.table_arena_bytes = d.table_arena_bytes;
     if (!c.host_threads) c.host_threads = d.host_threads;
+    if (!c.dma_piece_mib) c.dma_piece_mib = d.dma_piece_mib;
     auto* x = new aeg_ctx_s();
     try {
       x->c.init(device, c);

@@ -48,6 +48,16 @@ struct Xfer {
   bool failed = false;              // enqueue was interrupted by an error (events force-recorded)
   bool debug_done = false;          // host-only synthetic transfers
   uint64_t table_mark = 0;          // table-arena end offset to release on completion
+  // Swap-out only: its D2H of each layer is issued as `npiece` block-range pieces; piece p covers
+  // the transfer's blocks [piece_lo[p], piece_lo[p+1]) and pev[l * npiece + p] is recorded on the
+  // D2H stream right after piece p of layer l (stream order: pieces of a layer land in index
+  // order).  A swap-in reading those host blocks waits for the piece that wrote them instead of
+  // the whole layer (rule ❷ at sub-layer granularity), so a round trip's H2D of layer l starts
+  // one piece, not one layer, after the D2H of layer l began.
+  int32_t npiece = 0;
+  std::vector<int32_t> piece_lo;
+  std::vector<cudaEvent_t> pev;
+  std::unordered_map<aeg_block, int32_t> wpos;  // written host block -> its index in the transfer
 };
 
 // Device staging ring for one direction of KV swaps: a byte ring (slots x slot_bytes) in which

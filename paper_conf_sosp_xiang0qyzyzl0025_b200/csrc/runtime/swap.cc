@@ -80,6 +80,21 @@ std::vector<uint64_t> uniq(std::vector<uint64_t> v) {
   return v;
 }
 
+// Block-range pieces [a, b) of a segment for its host DMAs: a single-layer segment is cut into
+// balanced pieces of <= piece_bytes (sub-layer rule-❷ events, Xfer::pev); a multi-layer (packed)
+// segment stays one piece.
+std::vector<std::pair<int32_t, int32_t>> pieces_of(const Seg& g, uint64_t chunk, uint64_t piece_bytes) {
+  std::vector<std::pair<int32_t, int32_t>> out;
+  const int32_t m = g.i1 - g.i0;
+  const uint64_t bytes = uint64_t(m) * chunk;
+  int32_t np = 1;
+  if (g.lb - g.la == 1 && bytes > piece_bytes)
+    np = int32_t(std::min<uint64_t>(uint64_t(m), (bytes + piece_bytes - 1) / piece_bytes));
+  for (int32_t q = 0; q < np; ++q)
+    out.push_back({g.i0 + int32_t(int64_t(m) * q / np), g.i0 + int32_t(int64_t(m) * (q + 1) / np)});
+  return out;
+}
+
 }  // namespace
 
 // Copy-engine DMAs between a staging slot and the host blocks of segment g (layer-major staging
@@ -213,7 +228,26 @@ uint64_t Ctx::swap_out(const Shape& sh, const aeg_block* dev, const aeg_block* h
   const auto segs = plan(sh.L, n, sh.chunk(), ring_out.slot_bytes);
   const auto runs = runs_of(host, n);
   const uint64_t dstride = dp.lstride(sh);
+  const uint64_t piece_bytes = uint64_t(cfg.dma_piece_mib) << 20;
+  // sub-layer D2H pieces: the same block ranges in every layer (segments repeat per layer)
   for (const Seg& g : segs) {
+    if (g.la != 0) break;
+    if (g.lb != 1) break;  // packed small layers: per-layer events only
+    for (auto& pc : pieces_of(g, sh.chunk(), piece_bytes)) x->piece_lo.push_back(pc.first);
+  }
+  if (x->piece_lo.size() > 1) {
+    x->npiece = int32_t(x->piece_lo.size());
+    x->piece_lo.push_back(n);
+    x->pev.resize(size_t(sh.L) * size_t(x->npiece));
+    for (auto& e : x->pev) e = take_event(false);
+    x->wpos.reserve(size_t(n) * 2);
+    for (int32_t i = 0; i < n; ++i) x->wpos.emplace(host[i], i);
+  } else {
+    x->piece_lo.clear();
+  }
+  int32_t pidx = 0;
+  for (const Seg& g : segs) {
+    if (g.i0 == 0) pidx = 0;
     if (g.i0 == 0) wait_deps(s_gather, rdeps, g.la, g.lb);  // rule ❷
     cudaEvent_t full, freed;
     uint64_t roff;
@@ -239,9 +273,23 @@ uint64_t Ctx::swap_out(const Shape& sh, const aeg_block* dev, const aeg_block* h
     CUDA_TRY(cudaStreamWaitEvent(s_d2h, full, 0));
     tr_wait(s_d2h, full);
     if (g.i0 == 0) wait_deps(s_d2h, wdeps, g.la, g.lb);  // rule ❸
-    host_dmas(hp, host_kv, sh, runs, g, sp, cudaMemcpyDeviceToHost, s_d2h);
-    if (tracing)
-      tr("op d2h d2h r=" + ring_cells("SO", roff, seg_bytes) + " w=" + cells(1, hp, host, n, g.la, g.lb, g.i0, g.i1));
+    if (x->npiece > 1) {
+      for (auto& pc : pieces_of(g, sh.chunk(), piece_bytes)) {
+        const Seg sub{g.la, g.lb, pc.first, pc.second};
+        const uint64_t po = uint64_t(pc.first - g.i0) * sh.chunk();
+        host_dmas(hp, host_kv, sh, runs, sub, sp + po, cudaMemcpyDeviceToHost, s_d2h);
+        if (tracing)
+          tr("op d2h d2h r=" + ring_cells("SO", roff + po, uint64_t(pc.second - pc.first) * sh.chunk()) +
+             " w=" + cells(1, hp, host, n, g.la, g.lb, pc.first, pc.second));
+        cudaEvent_t pe = x->pev[size_t(g.la) * size_t(x->npiece) + size_t(pidx++)];
+        CUDA_TRY(cudaEventRecord(pe, s_d2h));
+        tr_record(s_d2h, pe);
+      }
+    } else {
+      host_dmas(hp, host_kv, sh, runs, g, sp, cudaMemcpyDeviceToHost, s_d2h);
+      if (tracing)
+        tr("op d2h d2h r=" + ring_cells("SO", roff, seg_bytes) + " w=" + cells(1, hp, host, n, g.la, g.lb, g.i0, g.i1));
+    }
     CUDA_TRY(cudaEventRecord(freed, s_d2h));
     tr_record(s_d2h, freed);
     if (g.i1 == n)
@@ -296,9 +344,27 @@ uint64_t Ctx::swap_in_from(const Shape& sh, int32_t peer, const aeg_block* host,
       for (int32_t i = 0; i < n; ++i) hp.deps_for_read(host[i], rdeps);
     for (int32_t i = 0; i < n; ++i) dp.deps_for_write(dev[i], wdeps);
   }
-  if (after) rdeps.push_back(after);  // rule ❷ across instances (Fig. 10 ③), per layer
   rdeps = uniq(rdeps);
   wdeps = uniq(wdeps);
+  // Rule ❷ at sub-layer granularity: host blocks last written by an in-flight swap-out of this
+  // context with D2H pieces are waited for per piece (the highest piece of that swap-out holding
+  // any block of our piece; its pieces land in order on one stream).  Other writers (and the
+  // cross-instance `after`): per-layer events.
+  std::vector<Xfer*> pdeps;
+  {
+    std::vector<uint64_t> rest;
+    for (uint64_t d : rdeps) {
+      auto it = xfers.find(d);
+      Xfer* w = it == xfers.end() ? nullptr : it->second.get();
+      if (w && w->kind == X_SWAP_OUT && w->npiece > 1 && w->L == sh.L && !w->failed && !w->complete.load())
+        pdeps.push_back(w);
+      else
+        rest.push_back(d);
+    }
+    rdeps.swap(rest);
+  }
+  if (after) rdeps.push_back(after);  // rule ❷ across instances (Fig. 10 ③), per layer
+  rdeps = uniq(rdeps);
   char *htab = nullptr, *dtab = nullptr;
   if (n > 0) {
     alloc_table(uint64_t(n) * 8, x->id, &htab, &dtab);
@@ -309,7 +375,32 @@ uint64_t Ctx::swap_in_from(const Shape& sh, int32_t peer, const aeg_block* host,
   const auto segs = plan(sh.L, n, sh.chunk(), ring_in.slot_bytes);
   const auto runs = runs_of(host, n);
   const uint64_t dstride = dp.lstride(sh);
+  const uint64_t piece_bytes = uint64_t(cfg.dma_piece_mib) << 20;
+  // per piece of a layer (same block ranges in every layer): (writer, its highest piece) to wait on
+  std::vector<std::vector<std::pair<Xfer*, int32_t>>> pneed;
+  if (!pdeps.empty()) {
+    for (const Seg& g : segs) {
+      if (g.la != 0) break;
+      for (auto& pc : pieces_of(g, sh.chunk(), piece_bytes)) {
+        std::vector<std::pair<Xfer*, int32_t>> need;
+        for (Xfer* w : pdeps) {
+          int32_t hi = -1;
+          for (int32_t i = pc.first; i < pc.second; ++i) {
+            auto f = w->wpos.find(host[i]);
+            if (f == w->wpos.end()) continue;
+            const int32_t p = int32_t(std::upper_bound(w->piece_lo.begin(), w->piece_lo.end(), f->second) -
+                                      w->piece_lo.begin()) - 1;
+            hi = std::max(hi, p);
+          }
+          if (hi >= 0) need.push_back({w, hi});
+        }
+        pneed.push_back(std::move(need));
+      }
+    }
+  }
+  int32_t pidx = 0;
   for (const Seg& g : segs) {
+    if (g.i0 == 0) pidx = 0;
     if (g.i0 == 0) wait_deps(s_h2d, rdeps, g.la, g.lb);  // rule ❷ per layer (reading 12)
     cudaEvent_t full, freed;
     uint64_t roff;
@@ -317,9 +408,27 @@ uint64_t Ctx::swap_in_from(const Shape& sh, int32_t peer, const aeg_block* host,
     const uint64_t seg_bytes = uint64_t(g.lb - g.la) * uint64_t(g.i1 - g.i0) * sh.chunk();
     char* sp = ring_in.acquire(seg_bytes, s_h2d, &full, &freed, &roff, tracing ? &waited : nullptr);
     for (cudaEvent_t e : waited) tr_wait(s_h2d, e);
-    host_dmas(hp, hbase, sh, runs, g, sp, cudaMemcpyHostToDevice, s_h2d);
-    if (tracing)
-      tr("op h2d h2d r=" + cells(1, hp, host, n, g.la, g.lb, g.i0, g.i1) + " w=" + ring_cells("SI", roff, seg_bytes));
+    if (!pneed.empty()) {
+      for (auto& pc : pieces_of(g, sh.chunk(), piece_bytes)) {
+        for (auto& nd : pneed[size_t(pidx)])
+          for (int32_t l = g.la; l < g.lb; ++l) {
+            cudaEvent_t e = nd.first->pev[size_t(l) * size_t(nd.first->npiece) + size_t(nd.second)];
+            CUDA_TRY(cudaStreamWaitEvent(s_h2d, e, 0));
+            tr_wait(s_h2d, e);
+          }
+        ++pidx;
+        const Seg sub{g.la, g.lb, pc.first, pc.second};
+        const uint64_t po = uint64_t(pc.first - g.i0) * sh.chunk();
+        host_dmas(hp, hbase, sh, runs, sub, sp + po, cudaMemcpyHostToDevice, s_h2d);
+        if (tracing)
+          tr("op h2d h2d r=" + cells(1, hp, host, n, g.la, g.lb, pc.first, pc.second) + " w=" +
+             ring_cells("SI", roff + po, uint64_t(pc.second - pc.first) * sh.chunk()));
+      }
+    } else {
+      host_dmas(hp, hbase, sh, runs, g, sp, cudaMemcpyHostToDevice, s_h2d);
+      if (tracing)
+        tr("op h2d h2d r=" + cells(1, hp, host, n, g.la, g.lb, g.i0, g.i1) + " w=" + ring_cells("SI", roff, seg_bytes));
+    }
     CUDA_TRY(cudaEventRecord(full, s_h2d));
     tr_record(s_h2d, full);
 

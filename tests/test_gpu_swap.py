@@ -152,6 +152,74 @@ def test_c1_swap_in_chained_on_swap_out_without_host_sync():
         ctx.shutdown()
 
 
+SHP = KVShape(2, 16, 64, 2, 16)           # Cl = 64 KiB: a 75-block layer (4.7 MiB) is never packed
+
+
+@pytest.mark.parametrize("host_layout", [aeg.LAYER_MAJOR, aeg.BLOCK_MAJOR])
+@pytest.mark.parametrize("slot", [2 << 20, 8 << 20])
+def test_swap_in_waits_per_d2h_piece(host_layout, slot):
+    """Rule ❷ at sub-layer granularity: with 1 MiB D2H pieces a swap-out's layer is
+    moved as several block-range pieces, each with its own event, and a chained swap-in waits for
+    the pieces holding its blocks instead of the whole layer.  The swap-in is issued while a gate
+    holds the swap-out back; the library's own primitive log must satisfy ❶❷❸ and the result must
+    equal the oracle (O5, O6) on every chunk.  slot = 2 MiB also splits each layer into segments."""
+    require_gpu()
+    import torch
+    MIB = 1 << 20
+    cfg = aeg.default_config(device_kv_bytes=32 * MIB, host_kv_bytes=24 * 1280 * KIB,
+                             dev_slab_bytes=MIB, host_slab_bytes=1280 * KIB,
+                             dev_slab_layout=aeg.LAYER_MAJOR, host_slab_layout=host_layout,
+                             staging_slot_bytes=slot, staging_slots=3, stage_ring_bytes=4 << 20,
+                             stage_chunk_bytes=1 << 20, device_weight_bytes=8 << 20, table_arena_bytes=4 << 20,
+                             host_threads=2, kernel=aeg.KERNEL_AUTO, dma_piece_mib=1)
+    ctx = aeg.Context(0, cfg)
+    dev = Side(ctx, aeg.POOL_DEVICE, cfg.device_kv_bytes, cfg.dev_slab_bytes, aeg.LAYER_MAJOR)
+    host = Side(ctx, aeg.POOL_HOST, cfg.host_kv_bytes, cfg.host_slab_bytes, host_layout)
+    try:
+        dev.poison(gi.TAG_NEVER)
+        host.poison(gi.TAG_NEVER)
+        dimg, himg = dev.poison_img(gi.TAG_NEVER), host.poison_img(gi.TAG_NEVER)
+        dc, do = requests(dev, dimg, SHP)
+        assert len(do) * SHP.chunk_bytes() > 4 * MIB
+        hc, ho = host.alloc(SHP, len(do))
+        s = torch.cuda.Stream()
+        gate = D.Gate()
+        gate.close_on(s.cuda_stream)
+        ctx.stream_fence(s.cuda_stream)
+        ctx.trace_enable(True)
+        x = ctx.kv_swap_out(SHP.as_tuple(), dc, hc, flags=aeg.FREE_SRC)
+        nc, no = dev.alloc(SHP, len(do))
+        xo = dev.oracle.begin(do)
+        dev.oracle.free(do)
+        # read the host blocks in reverse: the swap-in's first piece needs the swap-out's last one
+        y = ctx.kv_swap_in(SHP.as_tuple(), np.ascontiguousarray(hc[::-1]), nc)
+        assert not ctx.layer_ready(y, 0, aeg.READY_QUERY)
+        gate.open()
+        himg = OK.swap_out(dimg, dev.geom, himg, host.geom, SHP, do, ho)
+        exp = OK.swap_in(himg, host.geom, dimg, dev.geom, SHP, list(reversed(ho)), no)
+        cons = torch.cuda.Stream()
+        for l in range(SHP.L):
+            ctx.layer_ready(y, l, aeg.READY_WAIT_STREAM, cons.cuda_stream)
+        cons.synchronize()
+        ctx.layer_ready(y, -1, aeg.READY_BLOCK)
+        assert first_diff(dev.read(), exp) is None
+        assert first_diff(host.read(), himg) is None
+        dev.oracle.complete(xo)
+        text = ctx.trace_read()
+        log = parse_trace(text)
+        # the D2H of a layer is several ops (pieces), and the H2D waits before several ops per layer
+        d2h_ops = [e for e in log if e[0] == "op" and e[1] == "d2h"]
+        h2d_ops = [e for e in log if e[0] == "op" and e[1] == "h2d"]
+        assert len(d2h_ops) >= 5 * SHP.L and len(h2d_ops) >= 5 * SHP.L
+        log.append(("use", "u0x%x" % cons.cuda_stream,
+                    [f"D:{s}:{j}:{l}" for (s, j) in no for l in range(SHP.L)]))
+        assert check(log)
+        ctx.xfer_release(x)
+        ctx.xfer_release(y)
+    finally:
+        ctx.shutdown()
+
+
 def parse_trace(text):
     """Library trace lines -> oracle.rules log tuples."""
     log = []
