@@ -115,6 +115,7 @@ KV_SHAPES = {
     "llama-2-13b": (40, 40, 128, 2, 16),
     "qwen-1.8b": (24, 16, 128, 2, 16),
     "yi-9b": (48, 4, 128, 2, 16),
+    "yi-9b-tp4": (48, 1, 128, 2, 16),       # one KV head per rank: 8 KiB chunks
     "qwen-72b": (80, 64, 128, 2, 16),
     "qwen-72b-tp4": (80, 16, 128, 2, 16),
 }

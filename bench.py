@@ -1595,12 +1595,15 @@ def run_ours(args):
         else:
             c5 = {"skipped": "configs[4] is the 8-GPU TP=4 layout (one rank pair on 1 GPU); not defined for N=%d" % world}
         small = None if world > 1 else leg("small_chunk", lambda: small_chunk_leg(aeg, torch, kernel))
+        small_tp4 = None if world > 1 else leg("small_chunk_tp4",
+                                               lambda: small_chunk_leg(aeg, torch, kernel, model="yi-9b-tp4"))
         route = None if world > 1 else leg("host_route", lambda: host_route_leg(aeg, torch, kernel))
         alloc = leg("allocator", lambda: allocator_leg(aeg)) if rank == 0 else None
         cpu = None if args.no_cpu or rank != 0 else leg("cpu_baseline", cpu_baseline)
         out.update({"e2e": e2e, "verify": ver, "one_direction": one_dir, "pcie_memcpy_GBps": {k: round(v, 1) for k, v in pc.items()},
                     "switch": sw, "migrate": mig, "per_layer_overlap": ovl, "c5": c5, "allocator": alloc,
-                    "per_chunk_memcpy_baseline": base, "small_chunk": small, "host_route": route,
+                    "per_chunk_memcpy_baseline": base, "small_chunk": small, "small_chunk_tp4": small_tp4,
+                    "host_route": route,
                     "host": host_facts(),
                     "cpu_baseline": cpu})
         if not ver.get("ok"):

@@ -5,10 +5,12 @@ out like 8 layer-major 1 GiB slabs (one Qwen-7B layer of a slab = 32 MiB at offs
   1d_32m  : 256 x 32 MiB copies, host contiguous
   2d_layer: per layer one cudaMemcpy2DAsync (8 rows x 32 MiB, host pitch 1 GiB)  <- what swap.cc issues
   1d_layer: per layer 8 separate 32 MiB copies (same addresses as 2d_layer)
+  duplex share: a second direction started while an 8 GiB copy runs (GB/s it gets)
 Usage: python tools/dma_shape_probe.py"""
 import ctypes as C
 import json
 import sys
+import time
 
 import torch
 
@@ -66,6 +68,37 @@ def main():
                 best = max(best, 8 * GIB / (e0.elapsed_time(e1) * 1e6))
             out[f"{kn}_{name}"] = round(best, 2)
             print(kn, name, round(best, 2), flush=True)
+    # duplex share: an 8 GiB D2H stream is running when a 1 GiB H2D starts on another stream (and
+    # the reverse) -- GB/s each direction gets while both run (PCIe arbitration between posted
+    # writes (D2H) and read requests (H2D))
+    dev2 = torch.empty(GIB, dtype=torch.uint8, device="cuda")
+    s2 = torch.cuda.Stream()
+    hs2 = C.c_void_p(s2.cuda_stream)
+    for first, second in ((D2H, H2D), (H2D, D2H)):
+        torch.cuda.synchronize()
+        a0, a1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        b0, b1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        a0.record(s)
+        for q in range(8):
+            if first == D2H:
+                cp(hp + q * GIB, dp, GIB, D2H)
+            else:
+                cp(dp, hp + q * GIB, GIB, H2D)
+        a1.record(s)
+        # start the other direction once ~1 GiB of the first has moved
+        time.sleep(0.02)
+        b0.record(s2)
+        if second == H2D:
+            assert rt.cudaMemcpyAsync(C.c_void_p(dev2.data_ptr()), C.c_void_p(hp), C.c_size_t(GIB), H2D, hs2) == 0
+        else:
+            assert rt.cudaMemcpyAsync(C.c_void_p(hp), C.c_void_p(dev2.data_ptr()), C.c_size_t(GIB), D2H, hs2) == 0
+        b1.record(s2)
+        torch.cuda.synchronize()
+        kn = "d2h_running_then_h2d" if first == D2H else "h2d_running_then_d2h"
+        out[kn] = {"second_GBps": round(GIB / (b0.elapsed_time(b1) * 1e6), 2),
+                   "first_total_GBps": round(8 * GIB / (a0.elapsed_time(a1) * 1e6), 2),
+                   "second_started_ms": round(a0.elapsed_time(b0), 1)}
+        print(kn, out[kn], flush=True)
     json.dump(out, sys.stdout)
     print()
 
