@@ -220,6 +220,67 @@ def test_swap_in_waits_per_d2h_piece(host_layout, slot):
         ctx.shutdown()
 
 
+def test_swap_in_from_two_piecewise_swap_outs():
+    """One swap-in reads, in a shuffled order, half of the host blocks written by each of two
+    in-flight swap-outs that both used D2H pieces: before each of its H2D pieces it must wait for
+    the right piece of each writer (two piece dependencies, different highest pieces).  Gate-held,
+    checked by the happens-before checker on the library's log and against the oracle."""
+    require_gpu()
+    import torch
+    MIB = 1 << 20
+    cfg = aeg.default_config(device_kv_bytes=48 * MIB, host_kv_bytes=40 * MIB,
+                             dev_slab_bytes=MIB, host_slab_bytes=MIB,
+                             dev_slab_layout=aeg.BLOCK_MAJOR, host_slab_layout=aeg.LAYER_MAJOR,
+                             staging_slot_bytes=8 << 20, staging_slots=3, stage_ring_bytes=4 << 20,
+                             stage_chunk_bytes=1 << 20, device_weight_bytes=8 << 20, table_arena_bytes=4 << 20,
+                             host_threads=2, kernel=aeg.KERNEL_AUTO, dma_piece_mib=1)
+    ctx = aeg.Context(0, cfg)
+    dev = Side(ctx, aeg.POOL_DEVICE, cfg.device_kv_bytes, cfg.dev_slab_bytes, aeg.BLOCK_MAJOR)
+    host = Side(ctx, aeg.POOL_HOST, cfg.host_kv_bytes, cfg.host_slab_bytes, aeg.LAYER_MAJOR)
+    try:
+        dev.poison(gi.TAG_NEVER)
+        host.poison(gi.TAG_NEVER)
+        dimg, himg = dev.poison_img(gi.TAG_NEVER), host.poison_img(gi.TAG_NEVER)
+        batches = []
+        for m in (1, 2):
+            c, o = dev.alloc(SHP, 96)
+            fill_blocks(dev, dimg, SHP, o, [(0, j) for j in range(96)], m=m)
+            batches.append((c, o))
+        s = torch.cuda.Stream()
+        gate = D.Gate()
+        gate.close_on(s.cuda_stream)
+        ctx.stream_fence(s.cuda_stream)
+        ctx.trace_enable(True)
+        xs, hosts = [], []
+        for c, o in batches:
+            hc, ho = host.alloc(SHP, len(o))
+            xs.append(ctx.kv_swap_out(SHP.as_tuple(), c, hc))
+            hosts.append((hc, ho))
+        # half of each batch's host blocks, interleaved and shuffled
+        rng = np.random.default_rng(11)
+        pick = [(b, i) for b in (0, 1) for i in rng.choice(96, size=48, replace=False)]
+        pick = [pick[k] for k in rng.permutation(len(pick))]
+        hsel_c = np.array([hosts[b][0][i] for b, i in pick], dtype=np.uint64)
+        hsel_o = [hosts[b][1][i] for b, i in pick]
+        nc, no = dev.alloc(SHP, len(pick))
+        y = ctx.kv_swap_in(SHP.as_tuple(), hsel_c, nc)
+        assert not ctx.layer_ready(y, 0, aeg.READY_QUERY)
+        gate.open()
+        for (c, o), (hc, ho) in zip(batches, hosts):
+            himg = OK.swap_out(dimg, dev.geom, himg, host.geom, SHP, o, ho)
+        exp = OK.swap_in(himg, host.geom, dimg, dev.geom, SHP, hsel_o, no)
+        ctx.layer_ready(y, -1, aeg.READY_BLOCK)
+        for x in xs:
+            ctx.layer_ready(x, -1, aeg.READY_BLOCK)
+        assert first_diff(dev.read(), exp) is None
+        assert first_diff(host.read(), himg) is None
+        log = parse_trace(ctx.trace_read())
+        assert sum(1 for e in log if e[0] == "op" and e[1] == "h2d") >= 6 * SHP.L
+        assert check(log)
+    finally:
+        ctx.shutdown()
+
+
 def parse_trace(text):
     """Library trace lines -> oracle.rules log tuples."""
     log = []
