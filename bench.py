@@ -227,7 +227,7 @@ class SwapBench:
     tests/oracle_swapbench.py (test infrastructure)."""
 
     def __init__(self, aeg, sh, n_req, kernel, extra_host_slabs=8, weight_bytes=0, seed_cfg=2, slot_mib=0, slots=0,
-                 churn_slabs=12, dma_piece_mib=0):
+                 churn_slabs=12, dma_piece_mib=0, timing=True):
         import aeg_inputs as gi
         self.aeg, self.gi = aeg, gi
         self.sht = sh
@@ -244,7 +244,8 @@ class SwapBench:
         host_slabs = batch_slabs + extra_host_slabs
         self.seed = gi.kv_seed(seed_cfg)
         cfg = aeg.default_config(device_kv_bytes=dev_slabs * GIB, host_kv_bytes=host_slabs * GIB,
-                                 device_weight_bytes=weight_bytes, kernel=kernel, flags=aeg.CFG_TIMING)
+                                 device_weight_bytes=weight_bytes, kernel=kernel,
+                                 flags=aeg.CFG_TIMING if timing else 0)
         if slot_mib:
             cfg.staging_slot_bytes = slot_mib * MIB
         if slots:

@@ -555,7 +555,7 @@ void Ctx::launch(int kind, const CopyArgs& a, cudaStream_t s, int impl, int max_
   AEG_REQUIRE(e == cudaSuccess, AEG_ERR_CUDA, "copy kernel launch failed: %s", cudaGetErrorString(e));
   kstats[kind].launches++;
   kstats[kind].bytes += 2 * a.chunk * uint64_t(a.nl) * uint64_t(a.n);
-  if (timing) {
+  if (ta) {
     CUDA_TRY(cudaEventRecord(tb, s));
     pending_timing.push_back({kind, ta, tb});
     if (pending_timing.size() > 4096) resolve_timing(true);

@@ -370,7 +370,11 @@ uint64_t Ctx::swap_in_from(const Shape& sh, int32_t peer, const aeg_block* host,
     alloc_table(uint64_t(n) * 8, x->id, &htab, &dtab);
     uint64_t* t = reinterpret_cast<uint64_t*>(htab);
     for (int32_t i = 0; i < n; ++i) t[i] = dp.off0(dev[i], sh);
-    CUDA_TRY(cudaMemcpyAsync(dtab, htab, uint64_t(n) * 8, cudaMemcpyHostToDevice, s_scatter));
+    // uploaded on the H2D stream: every scatter waits for a `full` event recorded there after it.
+    // (A copy-engine op on the scatter stream made the scatters wait for the H2D stream to block
+    // on a ring slot whenever CUDA timing events bracket them — first layer of a chained round
+    // trip 89 ms instead of 40 ms, tools/roundtrip_timeline.py, profiles/r01/timeline.txt.)
+    CUDA_TRY(cudaMemcpyAsync(dtab, htab, uint64_t(n) * 8, cudaMemcpyHostToDevice, s_h2d));
   }
   const auto segs = plan(sh.L, n, sh.chunk(), ring_in.slot_bytes);
   const auto runs = runs_of(host, n);

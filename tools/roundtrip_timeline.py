@@ -18,12 +18,17 @@ def main():
     ap.add_argument("--dma-piece-mib", type=int, default=0)
     ap.add_argument("--requests", type=int, default=64)
     ap.add_argument("--reps", type=int, default=3)
+    ap.add_argument("--kernel", default="auto", choices=["auto", "lsu", "bulk"])
+    ap.add_argument("--slots", type=int, default=0)
+    ap.add_argument("--no-timing", action="store_true")
     a = ap.parse_args()
     import torch
     import bench
     import paper_conf_sosp_xiang0qyzyzl0025_b200 as aeg
     torch.cuda.init()
-    sb = bench.SwapBench(aeg, bench.QWEN7B, a.requests, aeg.KERNEL_AUTO, dma_piece_mib=a.dma_piece_mib).setup()
+    kern = {"auto": aeg.KERNEL_AUTO, "lsu": aeg.KERNEL_LSU, "bulk": aeg.KERNEL_BULK}[a.kernel]
+    sb = bench.SwapBench(aeg, bench.QWEN7B, a.requests, kern, dma_piece_mib=a.dma_piece_mib, slots=a.slots,
+                         timing=not a.no_timing).setup()
     ctx, sht, n, L = sb.ctx, sb.sht, sb.n, sb.L
     out = []
     for rep in range(a.reps):
@@ -52,7 +57,8 @@ def main():
         out.append({"enqueue_ms": [round((t1 - t0) * 1e3, 2), round((t2 - t1) * 1e3, 2)],
                     "swap_out_layer_ready_ms": [round(seen[(x, l)], 1) for l in range(L)],
                     "swap_in_layer_ready_ms": [round(seen[(y, l)], 1) for l in range(L)]})
-    print(json.dumps({"dma_piece_mib": sb.cfg.dma_piece_mib, "blocks": n, "runs": out}))
+    print(json.dumps({"dma_piece_mib": sb.cfg.dma_piece_mib, "kernel": a.kernel, "slots": sb.cfg.staging_slots,
+                      "timing": not a.no_timing, "blocks": n, "runs": out}))
     ctx.shutdown()
 
 
