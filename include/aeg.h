@@ -320,7 +320,10 @@ int aeg_export_ipc(aeg_ctx ctx, void* buf, uint64_t* len);
 int aeg_import_peer(aeg_ctx ctx, int32_t peer, const void* buf, uint64_t len);
 
 /* Serialise transfer x's per-layer interprocess events (after it was enqueued) so the peer can
- * wait on them; aeg_xfer_import turns such a blob into a local transfer id of the importer. */
+ * wait on them; aeg_xfer_import turns such a blob into a local transfer id of the importer.  A
+ * swap-out whose D2H ran in pieces (aeg_config.dma_piece_mib) also exports its per-(layer, piece)
+ * events, piece table and written host handles, so a peer's aeg_kv_swap_in_from(after = it) waits
+ * per piece (sub-layer rule ❷ across instances).  Call with buf = NULL to get the size. */
 int aeg_xfer_export(aeg_ctx ctx, aeg_xfer x, void* buf, uint64_t* len);
 int aeg_xfer_import(aeg_ctx ctx, int32_t peer, const void* buf, uint64_t len, aeg_xfer* out);
 

@@ -81,7 +81,19 @@ struct XferBlobHead {
   int32_t L;
   int32_t ipc;
   uint64_t id;
+  // swap-out D2H pieces (Xfer::pev), exported so a peer's swap-in waits per piece too: after the
+  // L + 1 layer/done handles come (npiece + 1) int32 piece starts, L * npiece event handles and the
+  // n written host handles in transfer order (0 pieces: nothing follows).
+  int32_t npiece;
+  int32_t n;
 };
+
+uint64_t xfer_blob_bytes(int32_t L, int32_t npiece, int32_t n) {
+  uint64_t b = sizeof(XferBlobHead) + uint64_t(L + 1) * sizeof(cudaIpcEventHandle_t);
+  if (npiece > 1)
+    b += uint64_t(npiece + 1) * 4 + uint64_t(L) * uint64_t(npiece) * sizeof(cudaIpcEventHandle_t) + uint64_t(n) * 8;
+  return b;
+}
 
 }  // namespace
 
@@ -539,25 +551,38 @@ int aeg_xfer_export(aeg_ctx ctx, aeg_xfer xid, void* buf, uint64_t* len) {
     std::lock_guard<std::mutex> g(c.mu);
     aeg::Xfer* x = c.get_xfer(xid);
     AEG_REQUIRE(x->done_recorded, AEG_ERR_STATE, "transfer not fully enqueued yet");
-    const uint64_t need = sizeof(XferBlobHead) + uint64_t(x->L + 1) * sizeof(cudaIpcEventHandle_t);
+    const int32_t np = x->npiece > 1 ? x->npiece : 0;
+    const int32_t nb = np ? int32_t(x->wpos.size()) : 0;
+    const uint64_t need = xfer_blob_bytes(x->L, np, nb);
     if (!buf) {
       *len = need;
       return AEG_OK;
     }
     AEG_REQUIRE(*len >= need, AEG_ERR_INVALID, "buffer too small");
     set_device(c);
-    XferBlobHead h{kXferMagic, int32_t(getpid()), x->L, x->ipc ? 1 : 0, x->id};
+    XferBlobHead h{kXferMagic, int32_t(getpid()), x->L, x->ipc ? 1 : 0, x->id, np, nb};
     char* o = static_cast<char*>(buf);
     std::memcpy(o, &h, sizeof h);
-    cudaIpcEventHandle_t* hs = reinterpret_cast<cudaIpcEventHandle_t*>(o + sizeof h);
-    for (int32_t l = 0; l <= x->L; ++l) {
-      cudaEvent_t e = l < x->L ? x->ev[l] : x->done_ev;
+    auto put_event = [&](cudaIpcEventHandle_t* hd, cudaEvent_t e) {
       if (x->ipc) {
-        CUDA_TRY(cudaIpcGetEventHandle(&hs[l], e));
+        CUDA_TRY(cudaIpcGetEventHandle(hd, e));
       } else {
-        std::memset(&hs[l], 0, sizeof hs[l]);
-        std::memcpy(&hs[l], &e, sizeof e);  // same-process peers use the event directly
+        std::memset(hd, 0, sizeof *hd);
+        std::memcpy(hd, &e, sizeof e);  // same-process peers use the event directly
       }
+    };
+    cudaIpcEventHandle_t* hs = reinterpret_cast<cudaIpcEventHandle_t*>(o + sizeof h);
+    for (int32_t l = 0; l <= x->L; ++l) put_event(&hs[l], l < x->L ? x->ev[l] : x->done_ev);
+    if (np) {
+      char* q = o + sizeof h + uint64_t(x->L + 1) * sizeof(cudaIpcEventHandle_t);
+      std::memcpy(q, x->piece_lo.data(), uint64_t(np + 1) * 4);
+      q += uint64_t(np + 1) * 4;
+      cudaIpcEventHandle_t* ps = reinterpret_cast<cudaIpcEventHandle_t*>(q);
+      for (size_t k = 0; k < x->pev.size(); ++k) put_event(&ps[k], x->pev[k]);
+      q += x->pev.size() * sizeof(cudaIpcEventHandle_t);
+      std::vector<aeg_block> hb(size_t(nb), 0);
+      for (auto& kv : x->wpos) hb[size_t(kv.second)] = kv.first;
+      std::memcpy(q, hb.data(), uint64_t(nb) * 8);
     }
     *len = need;
     return AEG_OK;
@@ -571,7 +596,8 @@ int aeg_xfer_import(aeg_ctx ctx, int32_t peer, const void* buf, uint64_t len, ae
     XferBlobHead h;
     std::memcpy(&h, buf, sizeof h);
     AEG_REQUIRE(h.magic == kXferMagic, AEG_ERR_INVALID, "not an aegkv transfer blob");
-    AEG_REQUIRE(len >= sizeof h + uint64_t(h.L + 1) * sizeof(cudaIpcEventHandle_t), AEG_ERR_INVALID, "blob truncated");
+    AEG_REQUIRE(h.L >= 0 && h.npiece >= 0 && h.n >= 0 && len >= xfer_blob_bytes(h.L, h.npiece, h.n),
+                AEG_ERR_INVALID, "blob truncated");
     const bool same = h.pid == int32_t(getpid());
     AEG_REQUIRE(same || h.ipc, AEG_ERR_INVALID, "transfer events are not interprocess-capable");
     std::lock_guard<std::mutex> g(c.mu);
@@ -590,24 +616,46 @@ int aeg_xfer_import(aeg_ctx ctx, int32_t peer, const void* buf, uint64_t len, ae
     x->owns_events = false;
     x->recorded.assign(h.L, 1);
     x->ev.resize(h.L);
-    for (int32_t l = 0; l <= h.L; ++l) {
+    auto get_event = [&](const cudaIpcEventHandle_t& hd) {
       cudaEvent_t e;
       if (same) {
-        std::memcpy(&e, &hs[l], sizeof e);
+        std::memcpy(&e, &hd, sizeof e);
       } else {
-        std::string key(reinterpret_cast<const char*>(&hs[l]), sizeof hs[l]);
+        std::string key(reinterpret_cast<const char*>(&hd), sizeof hd);
         auto f = P->events.find(key);
         if (f == P->events.end()) {
-          CUDA_TRY(cudaIpcOpenEventHandle(&e, hs[l]));
+          CUDA_TRY(cudaIpcOpenEventHandle(&e, hd));
           P->events.emplace(key, e);
         } else {
           e = f->second;
         }
       }
+      return e;
+    };
+    for (int32_t l = 0; l <= h.L; ++l) {
+      cudaEvent_t e = get_event(hs[l]);
       if (l < h.L)
         x->ev[l] = e;
       else
         x->done_ev = e;
+    }
+    if (h.npiece > 1) {
+      const char* q = static_cast<const char*>(buf) + sizeof h + uint64_t(h.L + 1) * sizeof(cudaIpcEventHandle_t);
+      x->piece_lo.resize(size_t(h.npiece) + 1);
+      std::memcpy(x->piece_lo.data(), q, uint64_t(h.npiece + 1) * 4);
+      q += uint64_t(h.npiece + 1) * 4;
+      AEG_REQUIRE(x->piece_lo.front() == 0 && x->piece_lo.back() == h.n &&
+                      std::is_sorted(x->piece_lo.begin(), x->piece_lo.end()),
+                  AEG_ERR_INVALID, "bad piece table in transfer blob");
+      const cudaIpcEventHandle_t* ps = reinterpret_cast<const cudaIpcEventHandle_t*>(q);
+      x->pev.resize(size_t(h.L) * size_t(h.npiece));
+      for (size_t k = 0; k < x->pev.size(); ++k) x->pev[k] = get_event(ps[k]);
+      q += x->pev.size() * sizeof(cudaIpcEventHandle_t);
+      std::vector<aeg_block> hb(size_t(h.n));
+      std::memcpy(hb.data(), q, uint64_t(h.n) * 8);
+      x->wpos.reserve(hb.size() * 2);
+      for (int32_t i = 0; i < h.n; ++i) x->wpos.emplace(hb[size_t(i)], i);
+      x->npiece = h.npiece;
     }
     x->done_recorded = true;
     *out = x->id;

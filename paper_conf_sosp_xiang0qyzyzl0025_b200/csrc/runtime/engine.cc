@@ -346,7 +346,7 @@ void Ctx::housekeeping() {
       if (x->owns_events && !host_only) {
         for (cudaEvent_t e : x->ev) give_event(e, x->ipc);
         if (x->done_ev) give_event(x->done_ev, x->ipc);
-        for (cudaEvent_t e : x->pev) give_event(e, false);
+        for (cudaEvent_t e : x->pev) give_event(e, x->ipc);
       }
       it = xfers.erase(it);
     } else {

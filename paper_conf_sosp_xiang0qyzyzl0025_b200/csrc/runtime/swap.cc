@@ -239,7 +239,7 @@ uint64_t Ctx::swap_out(const Shape& sh, const aeg_block* dev, const aeg_block* h
     x->npiece = int32_t(x->piece_lo.size());
     x->piece_lo.push_back(n);
     x->pev.resize(size_t(sh.L) * size_t(x->npiece));
-    for (auto& e : x->pev) e = take_event(false);
+    for (auto& e : x->pev) e = take_event(x->ipc);  // exportable with the layer events
     x->wpos.reserve(size_t(n) * 2);
     for (int32_t i = 0; i < n; ++i) x->wpos.emplace(host[i], i);
   } else {
@@ -305,6 +305,12 @@ uint64_t Ctx::swap_out(const Shape& sh, const aeg_block* dev, const aeg_block* h
 }
 
 // ------------------------------------------------------------------------------ swap-in H4
+// A writer whose D2H pieces a swap-in can wait on (its own swap-out, or a peer's imported one).
+static bool piecewise(const Xfer* w, int32_t L) {
+  return w && (w->kind == X_SWAP_OUT || w->kind == X_IMPORTED) && w->npiece > 1 && w->L == L && !w->failed &&
+         !w->complete.load();
+}
+
 uint64_t Ctx::swap_in(const Shape& sh, const aeg_block* host, const aeg_block* dev, int32_t n, uint32_t flags) {
   return swap_in_from(sh, -1, host, dev, n, 0, flags);
 }
@@ -356,14 +362,20 @@ uint64_t Ctx::swap_in_from(const Shape& sh, int32_t peer, const aeg_block* host,
     for (uint64_t d : rdeps) {
       auto it = xfers.find(d);
       Xfer* w = it == xfers.end() ? nullptr : it->second.get();
-      if (w && w->kind == X_SWAP_OUT && w->npiece > 1 && w->L == sh.L && !w->failed && !w->complete.load())
+      if (piecewise(w, sh.L))
         pdeps.push_back(w);
       else
         rest.push_back(d);
     }
     rdeps.swap(rest);
   }
-  if (after) rdeps.push_back(after);  // rule ❷ across instances (Fig. 10 ③), per layer
+  if (after) {  // rule ❷ across instances (Fig. 10 ③): per piece if the peer exported pieces
+    auto it = xfers.find(after);
+    if (it != xfers.end() && piecewise(it->second.get(), sh.L))
+      pdeps.push_back(it->second.get());
+    else
+      rdeps.push_back(after);
+  }
   rdeps = uniq(rdeps);
   char *htab = nullptr, *dtab = nullptr;
   if (n > 0) {

@@ -168,21 +168,21 @@ def test_two_process_ipc_migrate():
 
 
 # ------------------------------------------------------------------------------------ NEXT-2
-def _decode_side_host_route(conn):
+def _decode_side_host_route(conn, nslabs=4):
     try:
-        _decode_host_route_body(conn)
+        _decode_host_route_body(conn, nslabs)
     except BaseException:
         import traceback
         conn.send(("error", traceback.format_exc()))
         raise
 
 
-def _decode_host_route_body(conn):
+def _decode_host_route_body(conn, nslabs=4):
     """Decode instance of Fig. 10: imports the prefill instance's shared CPU cache and its swap-out
     events, swaps R1 in from there (C->D) without any host synchronisation on the prefill side's
     progress, and exports its swap-in so the prefill side can release the CPU blocks."""
     import sys
-    ctx, dev = make(aeg.LAYER_MAJOR, slab=MIB, nslabs=4)
+    ctx, dev = make(aeg.LAYER_MAJOR, slab=MIB, nslabs=nslabs)
     dev.poison(gi.TAG_NEVER)
     # connect once at start-up (mapping a peer's pool / registering its shared host region may wait
     # for the GPU to drain, so it must not sit on the critical path of a hand-off)
@@ -206,16 +206,20 @@ def _decode_host_route_body(conn):
     ctx.shutdown()
 
 
-def test_two_process_host_route_p_c_d():
+@pytest.mark.parametrize("nblocks", [20, 600])
+def test_two_process_host_route_p_c_d(nblocks):
     """NEXT-2: prefill P swaps R1 out to its part of the node-shared
     CPU KV cache (P->C) behind a 0.2 s delay kernel; decode D swaps it in (C->D) waiting only on P's
     per-layer IPC events (rule ❷); P frees the CPU blocks after importing D's swap-in, so they stay
-    in P's move list until D is done (rule ❸).  D's device image = oracle swap_in∘swap_out."""
+    in P's move list until D is done (rule ❸).  D's device image = oracle swap_in∘swap_out.
+    nblocks = 600: 4.7 MiB layers, so P's D2H runs in pieces whose IPC events travel in the
+    transfer blob and D's H2D waits per piece."""
     require_gpu()
     import torch
+    nslabs = 4 if nblocks <= 160 else 16
     ctxm = mp.get_context("spawn")
     parent, child = ctxm.Pipe()
-    p = ctxm.Process(target=_decode_side_host_route, args=(child,))
+    p = ctxm.Process(target=_decode_side_host_route, args=(child, nslabs))
     p.start()
     child.close()
 
@@ -227,19 +231,20 @@ def test_two_process_host_route_p_c_d():
         return m
 
     try:
-        cfg = aeg.default_config(device_kv_bytes=4 * MIB, host_kv_bytes=4 * MIB, dev_slab_bytes=MIB,
+        cfg = aeg.default_config(device_kv_bytes=nslabs * MIB, host_kv_bytes=nslabs * MIB, dev_slab_bytes=MIB,
                                  host_slab_bytes=MIB, host_slab_layout=aeg.BLOCK_MAJOR, staging_slot_bytes=MIB,
                                  staging_slots=2, stage_ring_bytes=4 * MIB, stage_chunk_bytes=MIB,
-                                 table_arena_bytes=2 * MIB, host_threads=1, flags=aeg.CFG_SHARED_HOST)
+                                 table_arena_bytes=2 * MIB, host_threads=1, flags=aeg.CFG_SHARED_HOST,
+                                 dma_piece_mib=1)
         a = aeg.Context(0, cfg)
-        A = Side(a, aeg.POOL_DEVICE, 4 * MIB, MIB, aeg.LAYER_MAJOR)
-        H = Side(a, aeg.POOL_HOST, 4 * MIB, MIB, aeg.BLOCK_MAJOR)
+        A = Side(a, aeg.POOL_DEVICE, nslabs * MIB, MIB, aeg.LAYER_MAJOR)
+        H = Side(a, aeg.POOL_HOST, nslabs * MIB, MIB, aeg.BLOCK_MAJOR)
         A.poison(gi.TAG_NEVER)
         H.poison(gi.TAG_NEVER)
         aimg, himg = A.poison_img(gi.TAG_NEVER), H.poison_img(gi.TAG_NEVER)
-        sc, so = A.alloc(SH, 20)
-        fill_blocks(A, aimg, SH, so, [(1, j) for j in range(20)])
-        hc, ho = H.alloc(SH, 20)
+        sc, so = A.alloc(SH, nblocks)
+        fill_blocks(A, aimg, SH, so, [(1, j) for j in range(nblocks)])
+        hc, ho = H.alloc(SH, nblocks)
         parent.send(a.export_ipc())                   # instances connect at start-up
         assert recv() == "ready"                      # the decode instance is up and connected
         s = torch.cuda.Stream()
@@ -248,7 +253,10 @@ def test_two_process_host_route_p_c_d():
         gate.close_on(s.cuda_stream)                  # the prefill is still running until gate.open()
         a.stream_fence(s.cuda_stream)
         xo = a.kv_swap_out(SH.as_tuple(), sc, hc, flags=aeg.FREE_SRC)                            # ①②
-        parent.send(([int(b) for b in hc], a.xfer_export(xo)))
+        xob = a.xfer_export(xo)
+        # 32-byte head + (L + 1) 64-byte IPC event handles; pieces add their table and events
+        assert (len(xob) > 32 + (SH.L + 1) * 64) == (nblocks * SH.chunk_bytes() > 4 * MIB)
+        parent.send(([int(b) for b in hc], xob))
         xblob, do = recv()
         xd = a.xfer_import(1, xblob)
         out_done = a.layer_ready(xo, -1, aeg.READY_QUERY)
@@ -256,12 +264,12 @@ def test_two_process_host_route_p_c_d():
         a.kv_free_after(aeg.POOL_HOST, hc, xd)        # Ry-style: CPU blocks wait in the move list
         q = a.stats(aeg.POOL_HOST).quarantined_blocks
         fresh = a.kv_alloc(aeg.POOL_HOST, SH.as_tuple(), 4)      # allocation skips them (❸)
-        assert (out_done, in_done, q) == (False, False, 20)
+        assert (out_done, in_done, q) == (False, False, nblocks)
         assert not {aeg.decode_block(b)[1:] for b in fresh} & set(map(tuple, ho))
         gate.open()                                   # prefill done: P->C runs, then C->D on D's side
         got = np.frombuffer(recv(), dtype=np.uint8)
         himg2 = OK.swap_out(aimg, A.geom, himg, H.geom, SH, so, ho)
-        geom = OK.PoolGeom(4 * MIB, MIB, aeg.LAYER_MAJOR)
+        geom = OK.PoolGeom(nslabs * MIB, MIB, aeg.LAYER_MAJOR)
         dimg = gi.region_bytes(gi.kv_seed(1), gi.poison_key(gi.TAG_NEVER, 0), geom.nbytes)
         exp = OK.swap_in(himg2, H.geom, dimg, geom, SH, ho, do)
         assert first_diff(got, exp) is None
