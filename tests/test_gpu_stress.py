@@ -31,14 +31,34 @@ def dec(bs):
 
 @pytest.mark.parametrize("seed", range(6))
 def test_random_overlapping_transfers(seed):
-    require_gpu()
-    import torch
-    r = random.Random(seed)
     cfg = aeg.default_config(device_kv_bytes=24 * 256 * KIB, host_kv_bytes=24 * 256 * KIB, dev_slab_bytes=256 * KIB,
                              host_slab_bytes=256 * KIB, dev_slab_layout=seed % 2, host_slab_layout=(seed // 2) % 2,
                              staging_slot_bytes=1 << 20, staging_slots=2, stage_ring_bytes=4 << 20,
                              stage_chunk_bytes=1 << 20, device_weight_bytes=2 << 20, table_arena_bytes=2 << 20,
                              host_threads=1, kernel=aeg.KERNEL_BULK if seed % 3 else aeg.KERNEL_LSU)
+    _stress(seed, cfg, SH, 12)
+
+
+SHB = KVShape(2, 32, 128, 2, 16)         # 256 KiB chunks: layers of >= 16 blocks are >= 4 MiB (pieces)
+
+
+@pytest.mark.parametrize("seed", range(4))
+def test_random_overlapping_transfers_with_d2h_pieces(seed):
+    """The same stress with 1 MiB D2H pieces and layers big enough to use them: swap-ins (and
+    migrates) of host blocks written by in-flight piecewise swap-outs wait per piece."""
+    cfg = aeg.default_config(device_kv_bytes=40 * 2048 * KIB, host_kv_bytes=40 * 2048 * KIB,
+                             dev_slab_bytes=2048 * KIB, host_slab_bytes=2048 * KIB, dev_slab_layout=seed % 2,
+                             host_slab_layout=(seed // 2) % 2, staging_slot_bytes=(4 << 20) if seed % 2 else (8 << 20),
+                             staging_slots=2, stage_ring_bytes=4 << 20, stage_chunk_bytes=1 << 20,
+                             device_weight_bytes=2 << 20, table_arena_bytes=2 << 20, host_threads=1,
+                             kernel=aeg.KERNEL_AUTO, dma_piece_mib=1)
+    _stress(100 + seed, cfg, SHB, 28, lo=14)
+
+
+def _stress(seed, cfg, SH, nmax, lo=1):
+    require_gpu()
+    import torch
+    r = random.Random(seed)
     ctx = aeg.Context(0, cfg)
     try:
         dev = Side(ctx, 0, cfg.device_kv_bytes, cfg.dev_slab_bytes, cfg.dev_slab_layout)
@@ -58,7 +78,7 @@ def test_random_overlapping_transfers(seed):
         for step in range(45):
             op = r.choice(["new", "new", "out", "out", "in", "in", "mig", "free", "gate", "open", "use"])
             if op == "new" or not objs:
-                n = r.randint(1, 12)
+                n = r.randint(lo, nmax)
                 try:
                     c = ctx.kv_alloc(0, SH.as_tuple(), n)
                 except aeg.AegError:
