@@ -52,7 +52,9 @@ def test_random_overlapping_transfers_with_d2h_pieces(seed):
                              staging_slots=2, stage_ring_bytes=4 << 20, stage_chunk_bytes=1 << 20,
                              device_weight_bytes=2 << 20, table_arena_bytes=2 << 20, host_threads=1,
                              kernel=aeg.KERNEL_AUTO, dma_piece_mib=1)
-    _stress(100 + seed, cfg, SHB, 28, lo=14)
+    log, n_out = _stress(100 + seed, cfg, SHB, 28, lo=14)
+    # the swap-outs really ran in pieces: more D2H ops than (swap-out, layer) pairs
+    assert n_out > 0 and sum(1 for e in log if e[0] == "op" and e[1] == "d2h") > n_out * SHB.L
 
 
 def _stress(seed, cfg, SH, nmax, lo=1):
@@ -73,6 +75,7 @@ def _stress(seed, cfg, SH, nmax, lo=1):
             log.extend(parse_trace(ctx.trace_read()))
 
         objs = []        # [where, handles]
+        n_out = 0
         gates = []       # open gates
         cons = torch.cuda.Stream()
         for step in range(45):
@@ -105,6 +108,7 @@ def _stress(seed, cfg, SH, nmax, lo=1):
                 if op == "out" and o[0] == "dev":
                     hc = ctx.kv_alloc(1, SH.as_tuple(), len(o[1]))
                     ctx.kv_swap_out(SH.as_tuple(), o[1], hc, flags=aeg.FREE_SRC)
+                    n_out += 1
                     himg = OK.swap_out(dimg, dev.geom, himg, host.geom, SH, dec(o[1]), dec(hc))
                     o[:] = ["host", hc]
                 elif op == "in" and o[0] == "host":
@@ -146,6 +150,7 @@ def _stress(seed, cfg, SH, nmax, lo=1):
         assert check(log)
         assert first_diff(dev.read(), dimg) is None
         assert first_diff(host.read(), himg) is None
+        return log, n_out
     finally:
         for g in locals().get("gates", []):
             g.open()
