@@ -507,6 +507,66 @@ def small_chunk_leg(aeg, torch, kernel, model="yi-9b", gib=1):
 
 
 
+def c1_leg(aeg, torch, kernel, reps=200):
+    """configs[0] (tiny: 2 layers, 4 KV heads, d=64, fp16, 16-token blocks, 8 requests <= 256
+    tokens, 75 blocks, 2.3 MiB) swap round trip: launch/latency-bound, so report the per-round-trip
+    latency (GPU: consumer-stream events from the fence to the swap-in's last layer; wall: the two
+    API calls + host sync) and the host enqueue time of each call.  Whole-image oracle parity of the
+    same workload: tests/test_gpu_swap.py.  Here: identity on every chunk after all round trips."""
+    import aeg_inputs as gi
+    from aeg_inputs import dev as D
+    sht = gi.KV_SHAPES["tiny"]
+    sh = aeg.KVShape.of(sht)
+    lens = gi.request_lengths(1, 8, 1, 256, forced=(1, 16, 17, 255, 256))
+    nb = sum(-(-t // 16) for t in lens)
+    kib = 1024
+    ctx = aeg.Context(0, aeg.default_config(device_kv_bytes=32 * 256 * kib, host_kv_bytes=32 * 256 * kib,
+                                            dev_slab_bytes=256 * kib, host_slab_bytes=256 * kib,
+                                            staging_slot_bytes=1 << 20, staging_slots=2, stage_ring_bytes=2 << 20,
+                                            stage_chunk_bytes=1 << 20, device_weight_bytes=2 << 20,
+                                            table_arena_bytes=2 << 20, host_threads=1, kernel=kernel))
+    dbase, _ = ctx.pool_region(0)
+    src = ctx.kv_alloc(0, sht, nb)
+    keys = np.array([gi.kv_key(1, 0, i, l) for i in range(nb) for l in range(sh.num_layers)], np.uint64)
+    seed = gi.kv_seed(1)
+    D.fill_chunks(dbase, chunk_offsets(ctx, 0, sht, src), keys, sh.chunk_bytes(), seed)
+    s = torch.cuda.Stream()
+    gpu_us, wall_us, enq_us = [], [], []
+    for it in range(reps + 10):
+        torch.cuda.synchronize()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        t0 = time.perf_counter()
+        e0.record(s)
+        ctx.stream_fence(s.cuda_stream)
+        hc = ctx.kv_alloc(1, sht, nb)
+        nd = ctx.kv_alloc(0, sht, nb)
+        t1 = time.perf_counter()
+        x = ctx.kv_swap_out(sht, src, hc, flags=aeg.FREE_SRC)
+        t2 = time.perf_counter()
+        y = ctx.kv_swap_in(sht, hc, nd, flags=aeg.FREE_SRC)
+        t3 = time.perf_counter()
+        ctx.layer_ready(y, -1, aeg.READY_WAIT_STREAM, s.cuda_stream)
+        e1.record(s)
+        e1.synchronize()
+        t4 = time.perf_counter()
+        ctx.layer_ready(x, -1, aeg.READY_BLOCK)
+        ctx.xfer_release(x)
+        ctx.xfer_release(y)
+        src = nd
+        if it >= 10:
+            gpu_us.append(e0.elapsed_time(e1) * 1e3)
+            wall_us.append((t4 - t0) * 1e6)
+            enq_us.append(((t2 - t1) * 1e6, (t3 - t2) * 1e6))
+    bad, _ = D.verify_chunks(dbase, chunk_offsets(ctx, 0, sht, src), keys, sh.chunk_bytes(), seed)
+    ctx.shutdown()
+    med = lambda v: round(statistics.median(v), 1)  # noqa: E731
+    return {"workload": f"configs[0] tiny KV, 8 requests ({nb} blocks, {nb * sh.block_bytes() / 2**20:.2f} MiB): "
+                        "swap-out + swap-in round trip, one at a time",
+            "round_trip_gpu_us_p50": med(gpu_us), "round_trip_wall_us_p50": med(wall_us),
+            "enqueue_us_p50": {"swap_out": med([a for a, _ in enq_us]), "swap_in": med([b for _, b in enq_us])},
+            "reps": reps, "bit_exact": bad == 0}
+
+
 def pcie_calibration(torch):
     """Plain cudaMemcpy of 1 GiB pinned <-> device: the copy engines' measured ceiling here."""
     h = torch.empty(GIB, dtype=torch.uint8, pin_memory=True)
@@ -1596,6 +1656,7 @@ def run_ours(args):
         else:
             c5 = {"skipped": "configs[4] is the 8-GPU TP=4 layout (one rank pair on 1 GPU); not defined for N=%d" % world}
         small = None if world > 1 else leg("small_chunk", lambda: small_chunk_leg(aeg, torch, kernel))
+        c1 = None if world > 1 else leg("c1", lambda: c1_leg(aeg, torch, kernel))
         small_tp4 = None if world > 1 else leg("small_chunk_tp4",
                                                lambda: small_chunk_leg(aeg, torch, kernel, model="yi-9b-tp4"))
         route = None if world > 1 else leg("host_route", lambda: host_route_leg(aeg, torch, kernel))
@@ -1603,7 +1664,7 @@ def run_ours(args):
         cpu = None if args.no_cpu or rank != 0 else leg("cpu_baseline", cpu_baseline)
         out.update({"e2e": e2e, "verify": ver, "one_direction": one_dir, "pcie_memcpy_GBps": {k: round(v, 1) for k, v in pc.items()},
                     "switch": sw, "migrate": mig, "per_layer_overlap": ovl, "c5": c5, "allocator": alloc,
-                    "per_chunk_memcpy_baseline": base, "small_chunk": small, "small_chunk_tp4": small_tp4,
+                    "per_chunk_memcpy_baseline": base, "small_chunk": small, "small_chunk_tp4": small_tp4, "c1": c1,
                     "host_route": route,
                     "host": host_facts(),
                     "cpu_baseline": cpu})
