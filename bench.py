@@ -871,15 +871,17 @@ def migrate_leg(aeg, torch, kernel, n_req=16, src_layout=None, dst_layout=None):
     doffs = chunk_offsets(b, 0, sht, dc)
     bad, _ = D.verify_chunks(bbase, doffs, keys, sh.chunk_bytes(), seed)
     # baseline on the same blocks: one cudaMemcpyAsync (copy engine, D2D) per (block, layer) chunk
+    # and the same chunks through cudaMemcpyBatchAsync: the copy-engine route with zero SMs
     s = torch.cuda.Stream()
-    bt = []
-    for _ in range(2):
-        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-        e0.record(s)
-        D.copy_chunks(bbase, doffs, abase, offs, sh.chunk_bytes(), s.cuda_stream)
-        e1.record(s)
-        e1.synchronize()
-        bt.append(e0.elapsed_time(e1))
+    bt, bb = [], []
+    for fn, acc in ((D.copy_chunks, bt), (D.copy_chunks_batch, bb)):
+        for _ in range(2):
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record(s)
+            fn(bbase, doffs, abase, offs, sh.chunk_bytes(), s.cuda_stream)
+            e1.record(s)
+            e1.synchronize()
+            acc.append(e0.elapsed_time(e1))
     a.shutdown()
     b.shutdown()
     payload = n * sh.block_bytes()
@@ -891,6 +893,7 @@ def migrate_leg(aeg, torch, kernel, n_req=16, src_layout=None, dst_layout=None):
             "kernel_ms_per_xfer": round(kms, 3), "bit_exact": bad == 0,
             "GBps_payload_by_ctas": sweep,
             "per_chunk_memcpy_baseline_GBps_payload": round(payload / (min(bt) * 1e6), 1),
+            "batch_api_ce_baseline_GBps_payload": round(payload / (min(bb) * 1e6), 1),
             "per_chunk_memcpy_calls": int(len(offs))}
 
 
@@ -998,6 +1001,36 @@ def migrate_leg_dist(aeg, torch, dist, kernel, n_req=16):
         keys = [gi.kv_key(1, sender, i, l) for i in range(n) for l in range(sh.num_layers)]
         bad, _ = D.verify_chunks(base, offs, keys, sh.chunk_bytes(), seed)
     bad = dist.sum(bad)
+    # CE-vs-SM: the same chunks paged -> paged through cudaMemcpyBatchAsync (copy
+    # engines, zero SMs) into the partner's pool mapped here (aeg_peer_region); decode ranks send
+    # their chunk offsets.  Max-over-ranks device time of one round, all pairs at once.
+    doffs_by_rank = PD.exchange(None if prefill else chunk_offsets(ctx, 0, sht, dst).tolist())
+    ce_err = []
+
+    def ce_round():
+        dist.barrier()
+        ms = 0.0
+        if prefill and not ce_err:
+            try:
+                d = [d_ for s_, d_ in pairs if s_ == rank][0]
+                pbase, _ = ctx.peer_region(d)
+                s = torch.cuda.Stream()
+                e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                e0.record(s)
+                D.copy_chunks_batch(pbase, np.asarray(doffs_by_rank[d], np.uint64), base, offs, sh.chunk_bytes(),
+                                    s.cuda_stream)
+                e1.record(s)
+                e1.synchronize()
+                ms = e0.elapsed_time(e1)
+            except Exception as e:  # noqa: BLE001  (every rank must still reach the max below)
+                ce_err.append(f"{type(e).__name__}: {e}")
+                ms = -1e9
+        return dist.max(ms)
+    ce_ms = min(ce_round() for _ in range(3))
+    failed = dist.sum(1 if ce_err else 0)
+    ce = ({"error": ce_err[0] if ce_err else "failed on another rank"} if failed or ce_ms <= 0 else
+          {"GBps_aggregate": round(len(pairs) * n * sh.block_bytes() / (ce_ms * 1e6), 1),
+           "what": "cudaMemcpyBatchAsync of the same (block, layer) chunks, copy engines only"})
     # SURVEY §8(d) C3 for N >= 4: all-to-all, every prefill rank -> every decode rank, round-robin
     a2a = None
     if world >= 4:
@@ -1012,7 +1045,7 @@ def migrate_leg_dist(aeg, torch, dist, kernel, n_req=16):
     ms = statistics.median(times)
     payload = len(pairs) * n * sh.block_bytes()
     return {"workload": f"configs[2] Llama-2-13B hand-off, {n_req} requests per pair, pairs {pairs}",
-            "nccl_sendrecv_contiguous_baseline": nccl,
+            "nccl_sendrecv_contiguous_baseline": nccl, "batch_api_ce_route": ce,
             "payload_bytes": payload, "ms": round(ms, 3), "GBps_aggregate": round(payload / (ms * 1e6), 1),
             "GBps_per_pair": round(payload / len(pairs) / (ms * 1e6), 1), "peak_per_direction_nominal": NVLINK_NOMINAL,
             "frac_of_nvlink_nominal_per_pair": round(payload / len(pairs) / (ms * 1e6) / NVLINK_NOMINAL, 3),

@@ -206,6 +206,11 @@ int aeg_block_offsets(aeg_ctx ctx, int32_t pool, const aeg_kv_shape* shape, cons
 /* Base pointer and size of a pool's region (device pointer for DEVICE, host pointer for HOST). */
 int aeg_pool_region(aeg_ctx ctx, int32_t pool, void** base, uint64_t* bytes);
 
+/* Base pointer (valid in this process: UVA / CUDA-IPC mapping) and size of the device KV region of
+ * an imported peer (aeg_import_peer index `peer`), for callers that address the peer's blocks
+ * themselves (e.g. a copy-engine comparison route).  AEG_ERR_INVALID if the peer was not imported. */
+int aeg_peer_region(aeg_ctx ctx, int32_t peer, void** base, uint64_t* bytes);
+
 /* ---- KV movement (H2-H6) ------------------------------------------------------------------ */
 
 /* Swap-out P->C (Fig. 10 steps ①②): for i < n and every layer l,

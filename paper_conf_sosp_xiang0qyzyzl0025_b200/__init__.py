@@ -98,6 +98,7 @@ _SIGS = {
     "aeg_block_info": [P, U64, PI32, PU32, PU32],
     "aeg_block_ptr": [P, I32, C.POINTER(KVShape), U64, I32, C.POINTER(P)],
     "aeg_pool_region": [P, I32, C.POINTER(P), PU64],
+    "aeg_peer_region": [P, I32, C.POINTER(P), PU64],
     "aeg_block_offsets": [P, I32, C.POINTER(KVShape), PU64, I32, PU64, PU64],
     "aeg_kv_swap_out": [P, C.POINTER(KVShape), PU64, PU64, I32, U32, PU64],
     "aeg_kv_swap_in": [P, C.POINTER(KVShape), PU64, PU64, I32, U32, PU64],
@@ -239,6 +240,11 @@ class Context:
     def pool_region(self, pool: int):
         p, n = P(), C.c_uint64()
         _chk(lib().aeg_pool_region(self.h, pool, C.byref(p), C.byref(n)))
+        return p.value or 0, n.value
+
+    def peer_region(self, peer: int):
+        p, n = P(), C.c_uint64()
+        _chk(lib().aeg_peer_region(self.h, int(peer), C.byref(p), C.byref(n)))
         return p.value or 0, n.value
 
     # -- H2-H6

@@ -264,6 +264,18 @@ int aeg_pool_region(aeg_ctx ctx, int32_t pool, void** base, uint64_t* bytes) {
   });
 }
 
+int aeg_peer_region(aeg_ctx ctx, int32_t peer, void** base, uint64_t* bytes) {
+  return guarded([&] {
+    Ctx& c = C(ctx);
+    std::lock_guard<std::mutex> g(c.mu);
+    auto it = c.peers.find(peer);
+    AEG_REQUIRE(it != c.peers.end() && it->second->valid, AEG_ERR_INVALID, "peer %d not imported", peer);
+    if (base) *base = it->second->dev_kv;
+    if (bytes) *bytes = it->second->geom.pool_bytes;
+    return AEG_OK;
+  });
+}
+
 int aeg_kv_swap_out(aeg_ctx ctx, const aeg_kv_shape* shape, const aeg_block* dev, const aeg_block* host, int32_t n,
                     uint32_t flags, aeg_xfer* out) {
   return guarded([&] {
