@@ -621,7 +621,29 @@ def host_facts():
         f["numa_nodes"] = len([d for d in os.listdir("/sys/devices/system/node") if d.startswith("node")])
     except OSError:
         pass
+    f["all_core_host_memcpy_GBps"] = host_memcpy_ceiling()
     return f
+
+
+def host_memcpy_ceiling(mib=256, reps=4):
+    """Context row: all-core host memcpy GB/s (one thread per core, each copying its
+    own 256 MiB buffer; NumPy releases the GIL), counting read + write bytes like the oracle's GB/s
+    counts payload only once per direction -- here payload bytes copied."""
+    import threading
+    n = os.cpu_count() or 1
+    bufs = [(np.ones(mib << 20, np.uint8), np.ones(mib << 20, np.uint8)) for _ in range(n)]
+
+    def work(a, b):
+        for _ in range(reps):
+            np.copyto(b, a)
+    ths = [threading.Thread(target=work, args=ab) for ab in bufs]
+    t0 = time.perf_counter()
+    for t in ths:
+        t.start()
+    for t in ths:
+        t.join()
+    dt = time.perf_counter() - t0
+    return round(n * reps * (mib << 20) / dt / 1e9, 1)
 
 
 def model_caches(names):
@@ -1525,6 +1547,9 @@ def cpu_baseline(blocks=128, min_s=10.0):
     src = od.alloc(sh, blocks)
     hb = oh.alloc(sh, blocks)
     reps, t = 0, 0.0
+    aff = os.sched_getaffinity(0) if hasattr(os, "sched_getaffinity") else None
+    if aff:   # one host core: the oracle's copies are single-threaded anyway
+        os.sched_setaffinity(0, {min(aff)})
     while (reps == 0 or t < min_s) and reps < 50:
         t0 = time.perf_counter()
         host = OK.swap_out(dev, dg, host, hg, sh, src, hb)
@@ -1532,6 +1557,8 @@ def cpu_baseline(blocks=128, min_s=10.0):
         dev = OK.swap_in(host, hg, dev, dg, sh, hb, dst)
         t += time.perf_counter() - t0
         reps += 1
+    if aff:
+        os.sched_setaffinity(0, aff)
     moved = 2 * blocks * sh.block_bytes() * reps
     return {"value": round(moved / t / 1e9, 3), "unit": "GB/s", "cores": 1, "kind": "oracle",
             "sample": f"{reps} x swap-out+swap-in of {blocks} Qwen-7B blocks ({blocks * sh.block_bytes() >> 20} MiB "
