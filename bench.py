@@ -227,7 +227,7 @@ class SwapBench:
     tests/oracle_swapbench.py (test infrastructure)."""
 
     def __init__(self, aeg, sh, n_req, kernel, extra_host_slabs=8, weight_bytes=0, seed_cfg=2, slot_mib=0, slots=0,
-                 churn_slabs=12, dma_piece_mib=0, timing=True):
+                 churn_slabs=12, dma_piece_mib=0, timing=True, dev_batches=2, host_batches=1):
         import aeg_inputs as gi
         self.aeg, self.gi = aeg, gi
         self.sht = sh
@@ -240,8 +240,8 @@ class SwapBench:
         self.k = GIB // self.sh.block_bytes()
         batch_slabs = -(-self.n // self.k)
         self.churn_slabs = churn_slabs
-        dev_slabs = 2 * batch_slabs + self.churn_slabs + 4
-        host_slabs = batch_slabs + extra_host_slabs
+        dev_slabs = dev_batches * batch_slabs + self.churn_slabs + 4
+        host_slabs = host_batches * batch_slabs + extra_host_slabs
         self.seed = gi.kv_seed(seed_cfg)
         cfg = aeg.default_config(device_kv_bytes=dev_slabs * GIB, host_kv_bytes=host_slabs * GIB,
                                  device_weight_bytes=weight_bytes, kernel=kernel,
@@ -387,6 +387,42 @@ class SwapBench:
         if record:
             self.ops.append((hc, nd))
         self.src_c = nd
+
+    def back_to_back(self, torch, cons, k=6):
+        """Round trips issued back to back with no host synchronisation between them: round trip
+        j+1's swap-out of the blocks round trip j swapped in waits per layer on j's events (rule ❷)
+        and its fresh blocks come from the pools (rule ❸), so the D2H of j+1 overlaps the H2D of j.
+        The host keeps at most two round trips in flight (pool capacity: 3 batches on the device,
+        2 in host memory).  Returns GB/s over PCIe (out + in) on the consumer stream's clock."""
+        aeg = self.aeg
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        torch.cuda.synchronize()
+        e0.record(cons)
+        self.ctx.stream_fence(cons.cuda_stream)
+        inflight = []
+        for j in range(k):
+            if len(inflight) == 2:
+                for t in inflight.pop(0):
+                    self.ctx.layer_ready(t, -1, aeg.READY_BLOCK)
+                    self.ctx.xfer_release(t)
+            hc = self.ctx.kv_alloc(aeg.POOL_HOST, self.sht, self.n)
+            nd = self.ctx.kv_alloc(aeg.POOL_DEVICE, self.sht, self.n)
+            x = self.ctx.kv_swap_out(self.sht, self.src_c, hc, flags=aeg.FREE_SRC)
+            y = self.ctx.kv_swap_in(self.sht, hc, nd, flags=aeg.FREE_SRC)
+            inflight.append((x, y))
+            self.src_c = nd
+        for xs in inflight:
+            for t in xs:
+                self.ctx.layer_ready(t, -1, aeg.READY_WAIT_STREAM, cons.cuda_stream)
+        e1.record(cons)
+        e1.synchronize()
+        for xs in inflight:
+            for t in xs:
+                self.ctx.layer_ready(t, -1, aeg.READY_BLOCK)
+                self.ctx.xfer_release(t)
+        ms = e0.elapsed_time(e1)
+        return {"round_trips": k, "ms": round(ms, 1), "GBps": round(2 * k * self.n * self.sh.block_bytes() / (ms * 1e6), 2),
+                "ms_per_round_trip": round(ms / k, 1)}
 
     def one_direction(self, torch, cons):
         """Diagnostic (not in `value`): swap-out alone, then swap-in alone, each to completion, with
@@ -1641,7 +1677,8 @@ def run_ours(args):
     value = total_bytes / (ms_total * 1e6)
     g = sb.ctx.kernel_stats(aeg.K_GATHER)
     s = sb.ctx.kernel_stats(aeg.K_SCATTER)
-    launches_all = int(dist.sum(g[0] + s[0]))
+    f = sb.ctx.kernel_stats(aeg.K_FETCH)   # the block-table fetch kernel of each transfer
+    launches_all = int(dist.sum(g[0] + s[0] + f[0]))
     hbm, hbm_src = peaks()
     # dominant kernel = gather (HBM bound): algorithmic bytes per launch / mean CUDA-event duration
     g_per_launch_bytes = g[1] / max(1, g[0])
@@ -1690,6 +1727,24 @@ def run_ours(args):
             ver["ranks_failed"] = int(dist.sum(0 if ver.get("ok") else 1))
             ver["ok"] = ver["ranks_failed"] == 0
         sb.ctx.shutdown()
+
+        def b2b():
+            import psutil
+            need = 2 * sb.n * sb.sh.block_bytes() + 12 * GIB   # second host batch + slack
+            if world > 1 or psutil.virtual_memory().available < need + 16 * GIB:
+                return None
+            bb = SwapBench(aeg, QWEN7B, n_req, kernel, dev_batches=3, host_batches=2, timing=False).setup()
+            try:
+                bb.back_to_back(torch, cons, 2)          # warm-up
+                r = bb.back_to_back(torch, cons, 6)
+                v = bb.verify()
+                r["bit_exact"] = bool(v.get("ok"))
+                r["what"] = ("configs[1] round trips back to back, no host sync between them (rules ❷❸ order "
+                             "them per layer); context sized for 2 in flight")
+                return r
+            finally:
+                bb.ctx.shutdown()
+        back2back = leg("back_to_back", b2b)
         if args.no_migrate:
             mig = None
         elif world > 1:
@@ -1724,7 +1779,7 @@ def run_ours(args):
         cpu = None if args.no_cpu or rank != 0 else leg("cpu_baseline", cpu_baseline)
         out.update({"e2e": e2e, "verify": ver, "one_direction": one_dir, "pcie_memcpy_GBps": {k: round(v, 1) for k, v in pc.items()},
                     "switch": sw, "migrate": mig, "per_layer_overlap": ovl, "c5": c5, "allocator": alloc,
-                    "per_chunk_memcpy_baseline": base, "small_chunk": small, "small_chunk_tp4": small_tp4, "c1": c1,
+                    "per_chunk_memcpy_baseline": base, "small_chunk": small, "small_chunk_tp4": small_tp4, "c1": c1, "back_to_back": back2back,
                     "host_route": route,
                     "host": host_facts(),
                     "cpu_baseline": cpu})

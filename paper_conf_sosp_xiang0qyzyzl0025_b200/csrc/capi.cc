@@ -680,7 +680,7 @@ int aeg_xfer_import(aeg_ctx ctx, int32_t peer, const void* buf, uint64_t len, ae
 int aeg_kernel_stats(aeg_ctx ctx, int32_t kind, uint64_t* launches, uint64_t* bytes, double* ms) {
   return guarded([&] {
     Ctx& c = C(ctx);
-    AEG_REQUIRE(kind >= 0 && kind < 4, AEG_ERR_INVALID, "bad kernel kind");
+    AEG_REQUIRE(kind >= 0 && kind < 5, AEG_ERR_INVALID, "bad kernel kind");
     std::lock_guard<std::mutex> g(c.mu);
     set_device(c);
     c.resolve_timing(true);

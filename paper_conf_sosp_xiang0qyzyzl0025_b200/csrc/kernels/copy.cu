@@ -11,6 +11,7 @@
 // Both are persistent: the grid is one wave (148 SMs x resident CTAs) striding over items.
 #include <cuda_runtime.h>
 
+#include <algorithm>
 #include <atomic>
 #include <cstdint>
 
@@ -255,6 +256,19 @@ cudaError_t launch_t(const CopyArgs& a, int impl, int max_ctas, cudaStream_t s) 
   return cudaGetLastError();
 }
 
+// Block-table fetch: the transfer's table is read by the GPU straight from the pinned host mirror
+// (zero-copy, ld.global.cv: never a stale cached line of host memory the CPU has rewritten) into
+// the device table arena, on the kernel stream that then uses it.  Not a cudaMemcpyAsync: a copy
+// engine serves H2D copies FIFO across streams, so a table upload queued behind a swap-in's
+// gigabytes of H2D held the next swap-out's first gather until they drained.
+__global__ void __launch_bounds__(256) fetch_table(uint2* __restrict__ dst, const uint2* src, uint64_t words) {
+  for (uint64_t w = uint64_t(blockIdx.x) * blockDim.x + threadIdx.x; w < words; w += uint64_t(gridDim.x) * blockDim.x) {
+    uint2 v;
+    asm volatile("ld.global.cv.v2.u32 {%0,%1}, [%2];" : "=r"(v.x), "=r"(v.y) : "l"(src + w));
+    dst[w] = v;
+  }
+}
+
 template <bool SP, bool DP>
 cudaError_t preload_t() {
   cudaFuncAttributes fa;
@@ -271,7 +285,18 @@ cudaError_t preload_t() {
 // Load every copy kernel into the current device's context now.  With CUDA's lazy module loading a
 // kernel's first launch loads its module and waits for the device; on the hot path that is both a
 // latency spike and a deadlock hazard when another kernel spin-waits (found by the gate tests).
+cudaError_t launch_fetch_table(void* dst, const void* src_host, uint64_t bytes, cudaStream_t s) {
+  const uint64_t words = bytes / 8;
+  if (words == 0) return cudaSuccess;
+  const uint64_t ctas = std::min<uint64_t>(64, (words + 255) / 256);
+  fetch_table<<<unsigned(ctas), 256, 0, s>>>(static_cast<uint2*>(dst), static_cast<const uint2*>(src_host), words);
+  return cudaGetLastError();
+}
+
 cudaError_t preload_kernels() {
+  cudaFuncAttributes fa0;
+  cudaError_t e0 = cudaFuncGetAttributes(&fa0, fetch_table);
+  if (e0 != cudaSuccess) return e0;
   cudaError_t e = preload_t<true, false>();
   if (e == cudaSuccess) e = preload_t<false, true>();
   if (e == cudaSuccess) e = preload_t<true, true>();

@@ -31,6 +31,10 @@ enum CopyImpl { IMPL_LSU = 1, IMPL_BULK = 2, IMPL_WARP = 3 };
 // (cp.async.bulk global->smem->global, mbarrier pipeline, one issuing thread per CTA).
 cudaError_t launch_copy(const CopyArgs& a, int impl, int max_ctas, cudaStream_t s);
 
+// Copy a block table (bytes, multiple of 8) from pinned, device-mapped host memory to device
+// memory with a small kernel on `s` (zero-copy reads; no copy engine).
+cudaError_t launch_fetch_table(void* dst, const void* src_host, uint64_t bytes, cudaStream_t s);
+
 // Load all copy kernels (and set the BULK shared-memory attribute) for the current device.
 cudaError_t preload_kernels();
 

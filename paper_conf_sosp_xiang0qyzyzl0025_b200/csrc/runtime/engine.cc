@@ -534,6 +534,13 @@ uint64_t Ctx::alloc_table(uint64_t bytes, uint64_t xid, char** host, char** dev)
 }
 
 // ----------------------------------------------------------------------- kernels + timing
+void Ctx::fetch_table(char* dev, const char* host, uint64_t bytes, cudaStream_t s) {
+  cudaError_t e = launch_fetch_table(dev, host, bytes, s);
+  AEG_REQUIRE(e == cudaSuccess, AEG_ERR_CUDA, "table fetch launch failed: %s", cudaGetErrorString(e));
+  kstats[4].launches++;
+  kstats[4].bytes += bytes;
+}
+
 void Ctx::launch(int kind, const CopyArgs& a, cudaStream_t s, int impl, int max_ctas) {
   cudaEvent_t ta = nullptr, tb = nullptr;
   if (timing) {

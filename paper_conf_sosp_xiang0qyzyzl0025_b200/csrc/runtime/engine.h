@@ -164,7 +164,7 @@ struct Ctx {
   std::vector<std::pair<char*, uint64_t>> registered;
 
   bool timing = false;
-  KStat kstats[4];
+  KStat kstats[5];   // gather, scatter, migrate, relocate, table fetch
   std::vector<TimingRec> pending_timing;
   std::vector<cudaEvent_t> timing_pool;
 
@@ -192,6 +192,7 @@ struct Ctx {
   void wait_deps(cudaStream_t s, const std::vector<uint64_t>& deps, int32_t la, int32_t lb);
   int layer_ready(uint64_t x, int32_t layer, int mode, cudaStream_t s);
   uint64_t alloc_table(uint64_t bytes, uint64_t xid, char** host, char** dev);
+  void fetch_table(char* dev, const char* host, uint64_t bytes, cudaStream_t s);  // table -> device, kernel
 
   // ---- kernels / timing
   void launch(int kind, const CopyArgs& a, cudaStream_t s, int impl, int max_ctas);

@@ -80,18 +80,39 @@ std::vector<uint64_t> uniq(std::vector<uint64_t> v) {
   return v;
 }
 
-// Block-range pieces [a, b) of a segment for its host DMAs: a single-layer segment is cut into
-// balanced pieces of <= piece_bytes (sub-layer rule-❷ events, Xfer::pev); a multi-layer (packed)
-// segment stays one piece.
-std::vector<std::pair<int32_t, int32_t>> pieces_of(const Seg& g, uint64_t chunk, uint64_t piece_bytes) {
+// Block-range pieces [a, b) of a segment for its host DMAs (sub-layer rule-❷ events, Xfer::pev).
+// A single-layer segment larger than piece_bytes is cut at host-run boundaries (maximal runs of
+// consecutive host blocks of one slab), grouping whole runs up to piece_bytes, so each piece stays
+// ONE copy-engine command where host_dmas can merge it (equal whole runs at a constant pitch): a
+// stream holds only ~1,000 pending copies before the enqueueing call blocks
+// (tools/queue_depth_probe.py), and balanced cuts through runs tripled the command count.  A run
+// longer than piece_bytes is split evenly.  A multi-layer (packed) segment stays one piece.
+std::vector<std::pair<int32_t, int32_t>> pieces_of(const Seg& g, uint64_t chunk, uint64_t piece_bytes,
+                                                   const std::vector<Run>& runs) {
   std::vector<std::pair<int32_t, int32_t>> out;
-  const int32_t m = g.i1 - g.i0;
-  const uint64_t bytes = uint64_t(m) * chunk;
-  int32_t np = 1;
-  if (g.lb - g.la == 1 && bytes > piece_bytes)
-    np = int32_t(std::min<uint64_t>(uint64_t(m), (bytes + piece_bytes - 1) / piece_bytes));
-  for (int32_t q = 0; q < np; ++q)
-    out.push_back({g.i0 + int32_t(int64_t(m) * q / np), g.i0 + int32_t(int64_t(m) * (q + 1) / np)});
+  if (g.lb - g.la != 1 || uint64_t(g.i1 - g.i0) * chunk <= piece_bytes) {
+    out.push_back({g.i0, g.i1});
+    return out;
+  }
+  const int32_t cap = int32_t(std::max<uint64_t>(1, piece_bytes / chunk));  // blocks per piece
+  int32_t a = g.i0;
+  for (const Run& r : runs) {
+    const int32_t s0 = std::max(r.i0, g.i0), e0 = std::min(r.i0 + r.m, g.i1);
+    if (s0 >= e0) continue;
+    if (e0 - s0 > cap) {  // a long run: close the open piece, split the run evenly
+      if (s0 > a) out.push_back({a, s0});
+      const int32_t np = (e0 - s0 + cap - 1) / cap;
+      for (int32_t q = 0; q < np; ++q)
+        out.push_back({s0 + int32_t(int64_t(e0 - s0) * q / np), s0 + int32_t(int64_t(e0 - s0) * (q + 1) / np)});
+      a = e0;
+      continue;
+    }
+    if (e0 - a > cap && s0 > a) {  // this run would overfill the open piece: close it before the run
+      out.push_back({a, s0});
+      a = s0;
+    }
+  }
+  if (a < g.i1) out.push_back({a, g.i1});
   return out;
 }
 
@@ -223,7 +244,7 @@ uint64_t Ctx::swap_out(const Shape& sh, const aeg_block* dev, const aeg_block* h
     alloc_table(uint64_t(n) * 8, x->id, &htab, &dtab);
     uint64_t* t = reinterpret_cast<uint64_t*>(htab);
     for (int32_t i = 0; i < n; ++i) t[i] = dp.off0(dev[i], sh);
-    CUDA_TRY(cudaMemcpyAsync(dtab, htab, uint64_t(n) * 8, cudaMemcpyHostToDevice, s_gather));
+    fetch_table(dtab, htab, uint64_t(n) * 8, s_gather);
   }
   const auto segs = plan(sh.L, n, sh.chunk(), ring_out.slot_bytes);
   const auto runs = runs_of(host, n);
@@ -233,7 +254,7 @@ uint64_t Ctx::swap_out(const Shape& sh, const aeg_block* dev, const aeg_block* h
   for (const Seg& g : segs) {
     if (g.la != 0) break;
     if (g.lb != 1) break;  // packed small layers: per-layer events only
-    for (auto& pc : pieces_of(g, sh.chunk(), piece_bytes)) x->piece_lo.push_back(pc.first);
+    for (auto& pc : pieces_of(g, sh.chunk(), piece_bytes, runs)) x->piece_lo.push_back(pc.first);
   }
   if (x->piece_lo.size() > 1) {
     x->npiece = int32_t(x->piece_lo.size());
@@ -274,7 +295,7 @@ uint64_t Ctx::swap_out(const Shape& sh, const aeg_block* dev, const aeg_block* h
     tr_wait(s_d2h, full);
     if (g.i0 == 0) wait_deps(s_d2h, wdeps, g.la, g.lb);  // rule ❸
     if (x->npiece > 1) {
-      for (auto& pc : pieces_of(g, sh.chunk(), piece_bytes)) {
+      for (auto& pc : pieces_of(g, sh.chunk(), piece_bytes, runs)) {
         const Seg sub{g.la, g.lb, pc.first, pc.second};
         const uint64_t po = uint64_t(pc.first - g.i0) * sh.chunk();
         host_dmas(hp, host_kv, sh, runs, sub, sp + po, cudaMemcpyDeviceToHost, s_d2h);
@@ -382,11 +403,10 @@ uint64_t Ctx::swap_in_from(const Shape& sh, int32_t peer, const aeg_block* host,
     alloc_table(uint64_t(n) * 8, x->id, &htab, &dtab);
     uint64_t* t = reinterpret_cast<uint64_t*>(htab);
     for (int32_t i = 0; i < n; ++i) t[i] = dp.off0(dev[i], sh);
-    // uploaded on the H2D stream: every scatter waits for a `full` event recorded there after it.
-    // (A copy-engine op on the scatter stream made the scatters wait for the H2D stream to block
-    // on a ring slot whenever CUDA timing events bracket them — first layer of a chained round
-    // trip 89 ms instead of 40 ms, tools/roundtrip_timeline.py, profiles/r01/timeline.txt.)
-    CUDA_TRY(cudaMemcpyAsync(dtab, htab, uint64_t(n) * 8, cudaMemcpyHostToDevice, s_h2d));
+    // fetched on the scatter stream by a kernel (no copy-engine op on a kernel stream: with CUDA
+    // timing events around the scatters one made every scatter wait for the H2D stream to block on
+    // a ring slot, profiles/r01/timeline.txt; and no H2D copy queued behind other transfers' DMAs)
+    fetch_table(dtab, htab, uint64_t(n) * 8, s_scatter);
   }
   const auto segs = plan(sh.L, n, sh.chunk(), ring_in.slot_bytes);
   const auto runs = runs_of(host, n);
@@ -397,7 +417,7 @@ uint64_t Ctx::swap_in_from(const Shape& sh, int32_t peer, const aeg_block* host,
   if (!pdeps.empty()) {
     for (const Seg& g : segs) {
       if (g.la != 0) break;
-      for (auto& pc : pieces_of(g, sh.chunk(), piece_bytes)) {
+      for (auto& pc : pieces_of(g, sh.chunk(), piece_bytes, runs)) {
         std::vector<std::pair<Xfer*, int32_t>> need;
         for (Xfer* w : pdeps) {
           int32_t hi = -1;
@@ -425,7 +445,7 @@ uint64_t Ctx::swap_in_from(const Shape& sh, int32_t peer, const aeg_block* host,
     char* sp = ring_in.acquire(seg_bytes, s_h2d, &full, &freed, &roff, tracing ? &waited : nullptr);
     for (cudaEvent_t e : waited) tr_wait(s_h2d, e);
     if (!pneed.empty()) {
-      for (auto& pc : pieces_of(g, sh.chunk(), piece_bytes)) {
+      for (auto& pc : pieces_of(g, sh.chunk(), piece_bytes, runs)) {
         for (auto& nd : pneed[size_t(pidx)])
           for (int32_t l = g.la; l < g.lb; ++l) {
             cudaEvent_t e = nd.first->pev[size_t(l) * size_t(nd.first->npiece) + size_t(nd.second)];
@@ -519,7 +539,7 @@ uint64_t Ctx::migrate(const Shape& sh, const aeg_block* src, int32_t peer, const
     uint64_t* t = reinterpret_cast<uint64_t*>(htab);
     for (int32_t i = 0; i < n; ++i) t[i] = dp.off0(src[i], sh);
     for (int32_t i = 0; i < n; ++i) t[n + i] = dg->off0(dst[i], sh);
-    CUDA_TRY(cudaMemcpyAsync(dtab, htab, uint64_t(n) * 16, cudaMemcpyHostToDevice, s_migrate));
+    fetch_table(dtab, htab, uint64_t(n) * 16, s_migrate);
   }
   // Layers per launch: every launch pays a fixed ~8-36 us, so pack layers up to a
   // target payload.  Same-device destinations copy at HBM speed (a 133 MiB layer is ~45 us): pack to
