@@ -76,6 +76,24 @@ def parse():
     return p.parse_args()
 
 
+_RAW_STREAMS = []
+
+
+def new_stream(torch):
+    """A dedicated CUDA stream.  torch.cuda.Stream() hands out pooled streams round-robin (32 per
+    priority), so a "new" stream can be an earlier one with work still queued behind it, which
+    silently corrupts event timings (the switch leg's landing probes read 270 ms for a layer that
+    landed at 1 ms).  Created once per call through the CUDA runtime torch already loaded."""
+    import ctypes as C
+    rt = C.CDLL("libcudart.so.12")
+    s = C.c_void_p()
+    rc = rt.cudaStreamCreateWithFlags(C.byref(s), 1)   # cudaStreamNonBlocking
+    if rc != 0:
+        raise RuntimeError(f"cudaStreamCreateWithFlags failed: {rc}")
+    _RAW_STREAMS.append(s)
+    return torch.cuda.ExternalStream(s.value)
+
+
 # ----------------------------------------------------------------------------------- plumbing
 def dist_env():
     world = int(os.environ.get("WORLD_SIZE", "1"))
@@ -367,7 +385,7 @@ class SwapBench:
         if first_layer is not None:   # diagnostics: host enqueue time of each call, swap-out layer 0 landed
             self.enqueue_ms = ((t1 - t0) * 1e3, (t2 - t1) * 1e3)
             if not hasattr(self, "diag_stream"):
-                self.diag_stream = torch.cuda.Stream()
+                self.diag_stream = new_stream(torch)
             self.ctx.layer_ready(x, 0, aeg.READY_WAIT_STREAM, self.diag_stream.cuda_stream)
             ex = torch.cuda.Event(enable_timing=True)
             ex.record(self.diag_stream)
@@ -472,7 +490,7 @@ def chunk_memcpy_baseline(aeg, torch, ctx, sht, src_blocks, reps=2):
     dbase, _ = ctx.pool_region(aeg.POOL_DEVICE)
     hbase, _ = ctx.pool_region(aeg.POOL_HOST)
     so, ho, no = (chunk_offsets(ctx, p, sht, b) for p, b in ((0, src_blocks), (1, hc), (0, nd)))
-    s = torch.cuda.Stream()
+    s = new_stream(torch)
     out = {}
     for fn, pre in ((D.copy_chunks, ""), (D.copy_chunks_batch, "batch_api_")):
         for name, args in (("d2h", (hbase, ho, dbase, so)), ("h2d", (dbase, no, hbase, ho))):
@@ -509,7 +527,7 @@ def small_chunk_leg(aeg, torch, kernel, model="yi-9b", gib=1):
     keys = np.array([gi.kv_key(3, 0, i, l) for i in range(n) for l in range(sh.num_layers)], np.uint64)
     seed = gi.kv_seed(4)
     D.fill_chunks(dbase, chunk_offsets(ctx, 0, sht, src), keys, sh.chunk_bytes(), seed)
-    s = torch.cuda.Stream()
+    s = new_stream(torch)
     res = {}
     for it in range(3):
         hc = ctx.kv_alloc(1, sht, n)
@@ -566,7 +584,7 @@ def c1_leg(aeg, torch, kernel, reps=200):
     keys = np.array([gi.kv_key(1, 0, i, l) for i in range(nb) for l in range(sh.num_layers)], np.uint64)
     seed = gi.kv_seed(1)
     D.fill_chunks(dbase, chunk_offsets(ctx, 0, sht, src), keys, sh.chunk_bytes(), seed)
-    s = torch.cuda.Stream()
+    s = new_stream(torch)
     gpu_us, wall_us, enq_us = [], [], []
     for it in range(reps + 10):
         torch.cuda.synchronize()
@@ -608,7 +626,7 @@ def pcie_calibration(torch):
     h = torch.empty(GIB, dtype=torch.uint8, pin_memory=True)
     d = torch.empty(GIB, dtype=torch.uint8, device="cuda")
     out = {}
-    s = torch.cuda.Stream()
+    s = new_stream(torch)
     for name, fn in (("h2d", lambda: d.copy_(h, non_blocking=True)), ("d2h", lambda: h.copy_(d, non_blocking=True))):
         with torch.cuda.stream(s):
             fn()
@@ -622,7 +640,7 @@ def pcie_calibration(torch):
     # both directions at once (the ceiling of the round-trip `value`): 3 x 1 GiB each way
     h2 = torch.empty(GIB, dtype=torch.uint8, pin_memory=True)
     d2 = torch.empty(GIB, dtype=torch.uint8, device="cuda")
-    s2 = torch.cuda.Stream()
+    s2 = new_stream(torch)
     torch.cuda.synchronize()
     e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     e0.record(s)
@@ -744,7 +762,7 @@ def switch_leg(aeg, torch, n_switch, kernel, descs, mode="staged", caches=None, 
         ctx.weights_reset(-(-wsize[cur] // 256) * 256)
         o, xp = ctx.weights_stage(descs[names[1]])
         pre = (names[1], xp, int(o[0]), o)
-    cons = torch.cuda.Stream()
+    cons = new_stream(torch)
     res = []
     diag_ms = None
     order = [names[(i + 1) % len(names)] for i in range(n_switch + 3)]
@@ -785,7 +803,7 @@ def switch_leg(aeg, torch, n_switch, kernel, descs, mode="staged", caches=None, 
             if xo is None:
                 del probes["kv_out_all"]
             for name, (xx, l) in probes.items():
-                ds = torch.cuda.Stream()
+                ds = new_stream(torch)
                 ctx.layer_ready(xx, l, aeg.READY_WAIT_STREAM, ds.cuda_stream)
                 de = torch.cuda.Event(enable_timing=True)
                 de.record(ds)
@@ -809,7 +827,7 @@ def switch_leg(aeg, torch, n_switch, kernel, descs, mode="staged", caches=None, 
             ctx.stream_fence(cons.cuda_stream)
             xo = a_kv_out()
             if diag:
-                ds = torch.cuda.Stream()
+                ds = new_stream(torch)
                 ctx.layer_ready(xo, -1, aeg.READY_WAIT_STREAM, ds.cuda_stream)
                 de = torch.cuda.Event(enable_timing=True)
                 de.record(ds)
@@ -905,7 +923,7 @@ def migrate_leg(aeg, torch, kernel, n_req=16, src_layout=None, dst_layout=None):
         out = []
         for it in range(reps + 2):
             a.kernel_stats_reset()
-            s = torch.cuda.Stream()
+            s = new_stream(torch)
             e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
             e0.record(s)
             a.stream_fence(s.cuda_stream)
@@ -930,7 +948,7 @@ def migrate_leg(aeg, torch, kernel, n_req=16, src_layout=None, dst_layout=None):
     bad, _ = D.verify_chunks(bbase, doffs, keys, sh.chunk_bytes(), seed)
     # baseline on the same blocks: one cudaMemcpyAsync (copy engine, D2D) per (block, layer) chunk
     # and the same chunks through cudaMemcpyBatchAsync: the copy-engine route with zero SMs
-    s = torch.cuda.Stream()
+    s = new_stream(torch)
     bt, bb = [], []
     for fn, acc in ((D.copy_chunks, bt), (D.copy_chunks_batch, bb)):
         for _ in range(2):
@@ -1021,7 +1039,7 @@ def migrate_leg_dist(aeg, torch, dist, kernel, n_req=16):
         ms = 0.0
         xs = {}
         if prefill:
-            s = torch.cuda.Stream()
+            s = new_stream(torch)
             e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
             e0.record(s)
             ctx.stream_fence(s.cuda_stream)
@@ -1072,7 +1090,7 @@ def migrate_leg_dist(aeg, torch, dist, kernel, n_req=16):
             try:
                 d = [d_ for s_, d_ in pairs if s_ == rank][0]
                 pbase, _ = ctx.peer_region(d)
-                s = torch.cuda.Stream()
+                s = new_stream(torch)
                 e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
                 e0.record(s)
                 D.copy_chunks_batch(pbase, np.asarray(doffs_by_rank[d], np.uint64), base, offs, sh.chunk_bytes(),
@@ -1146,7 +1164,7 @@ def _host_route_decode(conn, n_req):
         ctx.import_peer(0, conn.recv())
         _dbg("D: peer imported")
         t = torch.zeros(1, dtype=torch.int64, device="cuda")
-        s = torch.cuda.Stream()
+        s = new_stream(torch)
         D.stamp(t.data_ptr(), s.cuda_stream)   # load every kernel now: a module load later would wait
         s.synchronize()                        # behind P's gate kernel
         conn.send("ready")
@@ -1216,7 +1234,7 @@ def host_route_leg(aeg, torch, kernel, n_req=4, reps=4):
         if recv() != "ready":
             raise RuntimeError("decode process handshake")
         ts = torch.zeros(2, dtype=torch.int64, device="cuda")
-        s, s2 = torch.cuda.Stream(), torch.cuda.Stream()
+        s, s2 = new_stream(torch), new_stream(torch)
         gate = D.Gate()
         for _ in range(reps + 1):
             hc = a.kv_alloc(1, sht, n)
@@ -1392,7 +1410,7 @@ def c5_leg(aeg, torch, kernel, dist=None, tp_rank=1, tp_size=4, reps=3, model="q
     def one(do_w, do_kv):
         if dist is not None:
             dist.barrier()
-        s = torch.cuda.Stream()
+        s = new_stream(torch)
         e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         e0.record(s)
         xw = xk = None
@@ -1534,7 +1552,7 @@ def overlap_leg(aeg, torch, kernel, work_us=500, reps=5):
     out = {}
     try:
         hb = ctx.kv_alloc(aeg.POOL_HOST, sh, n)
-        cons = torch.cuda.Stream()
+        cons = new_stream(torch)
         for mode in ("per_layer", "whole"):
             ts = []
             for _ in range(reps):
@@ -1651,7 +1669,7 @@ def run_ours(args):
                    dma_piece_mib=args.dma_piece_mib,
                    churn_slabs=args.churn_slabs).setup()
     sb.sink = torch.zeros(1, dtype=torch.int64, device="cuda")
-    cons = torch.cuda.Stream()
+    cons = new_stream(torch)
     bytes_step = 2 * sb.n * sb.sh.block_bytes()
     log(f"[rank {rank}] C2: {sb.n} blocks ({sb.n * sb.sh.block_bytes() / GIB:.2f} GiB), ctx init {sb.init_s:.1f} s")
     for _ in range(args.warmup):

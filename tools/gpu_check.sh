@@ -15,7 +15,7 @@ if [[ $what == *bench* ]]; then
 fi
 if [[ $what == *ncu* ]]; then
   timeout 900 ncu --metrics gpu__time_duration.sum,dram__bytes_read.sum,dram__bytes_write.sum --clock-control none \
-      -k regex:copy_ -c 400 --csv --log-file gpurun_out/ncu_fullsize_launches.csv \
+      -k regex:"copy_|fetch_table" -c 400 --csv --log-file gpurun_out/ncu_fullsize_launches.csv \
       python bench.py --profile --steps 1 --warmup 1 > gpurun_out/ncu_fullsize.log 2>&1
   echo "ncu rc=$?" >> gpurun_out/ncu_fullsize.log
 fi
