@@ -43,6 +43,7 @@ GIB = 1 << 30
 MIB = 1 << 20
 PCIE_NOMINAL = 64.0   # GB/s per direction, PCIe Gen5 x16
 NVLINK_NOMINAL = 900.0
+NVLINK_PEER_COPY = 770.0   # GB/s per direction, measured peer copy (B200_PROFILING.md)
 HBM_FALLBACK = 6650.0
 BETA = 0.625          # PAPER.md:2515 (Eq. 4)
 
@@ -1125,6 +1126,7 @@ def migrate_leg_dist(aeg, torch, dist, kernel, n_req=16):
             "payload_bytes": payload, "ms": round(ms, 3), "GBps_aggregate": round(payload / (ms * 1e6), 1),
             "GBps_per_pair": round(payload / len(pairs) / (ms * 1e6), 1), "peak_per_direction_nominal": NVLINK_NOMINAL,
             "frac_of_nvlink_nominal_per_pair": round(payload / len(pairs) / (ms * 1e6) / NVLINK_NOMINAL, 3),
+            "frac_of_measured_peer_copy_per_pair": round(payload / len(pairs) / (ms * 1e6) / NVLINK_PEER_COPY, 3),
             "kernel_GBps_payload_max_rank": round(k_gbps, 1), "kernel_launches_per_xfer": int(kl // 5) if kl else 0,
             "GBps_aggregate_by_ctas": sweep,
             "bit_exact": bad == 0, "all_to_all": a2a}
