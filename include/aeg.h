@@ -117,7 +117,10 @@ typedef struct {
                                    sysfs; unbound if unknown), n > 0 = node n-1, -1 = no binding */
   uint32_t dma_piece_mib;       /* swap-out D2H piece (MiB) for sub-layer rule-❷ waits of a
                                    chained swap-in; 0 = 128, >= 4096 = one piece
-                                   per segment (per-layer events only)                          */
+                                   per segment (per-layer events only).  Pieces are cut at host-run
+                                   boundaries; very small pieces on big transfers can exceed the
+                                   ~1,000 pending copies a stream holds, and the data call then
+                                   blocks until the copy engine drains (correct, not async)      */
   uint32_t reserved[5];
 } aeg_config;
 
