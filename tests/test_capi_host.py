@@ -171,6 +171,15 @@ def test_error_codes_and_validation():
     assert e.value.code == aeg.ERR_STATE
     assert "host-only" in aeg.lib().aeg_last_error().decode()
     assert len(c.kv_alloc(aeg.POOL_DEVICE, A, 0)) == 0
+    with pytest.raises(aeg.AegError) as e:
+        c.peer_region(3)                                 # never imported
+    assert e.value.code == aeg.ERR_INVALID
+    with pytest.raises(aeg.AegError) as e:
+        c.kernel_stats(5)                                # kinds 0..4 (4 = block-table fetch)
+    assert e.value.code == aeg.ERR_INVALID
+    assert c.kernel_stats(aeg.K_FETCH)[0] == 0
+    cfg = aeg.default_config()
+    assert cfg.dma_piece_mib == 128                      # sub-layer D2H pieces on by default
     c.shutdown()
 
 
