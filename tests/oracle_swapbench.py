@@ -109,3 +109,23 @@ class OracleSwapBench(bench.SwapBench):
                 "host_chunks_checked": int(known.size), "host_bad_words": int(hbad),
                 "numpy_sampled_chunks": 8, "numpy_sampled_bad_bytes": sample_bad,
                 "ok": bad_total == 0 and hbad == 0 and sample_bad == 0}
+
+    def replay_given_and_verify(self, ops):
+        """Oracle replay of round trips whose placements the library chose (ops = [(src, hc, nd)]
+        library handles, in host issue order) — for round trips issued back to back, where which
+        reclaimed blocks an allocation gets depends on GPU progress.  Sequential replay in host
+        order is the result rules ❷❸ must produce however the transfers overlapped.  Checks every
+        chunk of the device pool and every host chunk written."""
+        aeg, sh = self.aeg, self.osh
+        dec = lambda bs: [(s, j) for _, s, j in map(aeg.decode_block, bs)]  # noqa: E731
+        for src, hc, nd in ops:
+            self.hlab = OK.swap_out(self.lab, self.dg, self.hlab, self.hg, sh, dec(src), dec(hc), unit=self.Cl)
+            self.lab = OK.swap_in(self.hlab, self.hg, self.lab, self.dg, sh, dec(hc), dec(nd), unit=self.Cl)
+        cells = self.lab.size
+        bad_total = self._verify(self.dbase, np.arange(cells, dtype=np.uint64) * np.uint64(self.Cl), self.lab)
+        known = np.nonzero(self.hlab)[0]
+        hbad = self._verify(self.hbase, known.astype(np.uint64) * np.uint64(self.Cl), self.hlab[known])
+        return {"device_chunks_checked": int(cells), "device_bad_words": int(bad_total),
+                "host_chunks_checked": int(known.size), "host_bad_words": int(hbad),
+                "ok": bad_total == 0 and hbad == 0}
+

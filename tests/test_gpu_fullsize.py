@@ -37,6 +37,44 @@ def test_c2_full_size_round_trip():
         sb.ctx.shutdown()
 
 
+def test_c2_full_size_back_to_back():
+    """The bench's back_to_back leg at full size: six 31 GiB round trips issued with no host sync
+    between them (two in flight, no timing events), each swap-out reading blocks the previous
+    swap-in is still writing (rule ❷ per layer / piece) into host blocks the previous swap-in may
+    still read (❸).  The oracle replays the same placements sequentially; every chunk of the
+    device pool (~450k) and every written host chunk must match."""
+    require_gpu()
+    import torch
+    import bench
+    from .oracle_swapbench import OracleSwapBench
+    sb = OracleSwapBench(aeg, bench.QWEN7B, 64, aeg.KERNEL_AUTO, dev_batches=3, host_batches=2,
+                         timing=False).setup()
+    try:
+        ops, inflight = [], []
+        for j in range(6):
+            if len(inflight) == 2:
+                for t in inflight.pop(0):
+                    sb.ctx.layer_ready(t, -1, aeg.READY_BLOCK)
+                    sb.ctx.xfer_release(t)
+            hc = sb.ctx.kv_alloc(aeg.POOL_HOST, sb.sht, sb.n)
+            nd = sb.ctx.kv_alloc(aeg.POOL_DEVICE, sb.sht, sb.n)
+            x = sb.ctx.kv_swap_out(sb.sht, sb.src_c, hc, flags=aeg.FREE_SRC)
+            y = sb.ctx.kv_swap_in(sb.sht, hc, nd, flags=aeg.FREE_SRC)
+            inflight.append((x, y))
+            ops.append((sb.src_c, hc, nd))
+            sb.src_c = nd
+        for xs in inflight:
+            for t in xs:
+                sb.ctx.layer_ready(t, -1, aeg.READY_BLOCK)
+                sb.ctx.xfer_release(t)
+        torch.cuda.synchronize()
+        v = sb.replay_given_and_verify(ops)
+        assert v["device_chunks_checked"] > 400_000 and v["host_chunks_checked"] >= 2 * sb.n * 32, v
+        assert v["ok"], v
+    finally:
+        sb.ctx.shutdown()
+
+
 def test_qwen18b_tp2_weights_full_size_sampled():
     require_gpu()
     descs_all = gi.model_tensors("qwen-1.8b")
