@@ -344,7 +344,7 @@ int aeg_set_migrate_ctas(aeg_ctx ctx, int32_t ctas);
 /* ---- instrumentation ---------------------------------------------------------------------- */
 
 /* Kernel counters since the last reset (needs AEG_CFG_TIMING for ms): kind 0 gather, 1 scatter,
- * 2 migrate, 3 relocate, 4 block-table fetch (launches and table bytes only, never timed).
+ * 2 migrate, 3 relocate, 4 block-table fetch (3 and 4: launches and bytes only, never timed).
  * launches / algorithmic bytes moved (payload read + written) / summed CUDA-event ms of the
  * launches (each timed on its own stream). */
 int aeg_kernel_stats(aeg_ctx ctx, int32_t kind, uint64_t* launches, uint64_t* bytes, double* ms);

@@ -595,18 +595,12 @@ uint64_t Ctx::relocate(uint64_t src_off, uint64_t dst_off, uint64_t bytes) {
               "relocation offsets and size must be multiples of 16");
   Xfer* x = new_xfer(X_RELOCATE, 1, false);
   int nl = 0;
-  cudaEvent_t ta = nullptr, tb = nullptr;
-  if (timing) {
-    CUDA_TRY(cudaEventCreate(&ta));
-    CUDA_TRY(cudaEventCreate(&tb));
-    CUDA_TRY(cudaEventRecord(ta, s_weights));
-  }
+  // Not bracketed by CUDA timing events even under AEG_CFG_TIMING: the weights stream also carries
+  // copy-engine DMAs, and timing events on a stream that mixes copy-engine ops and kernels held the
+  // kernel until other streams' queued H2D drained — a switch's relocation would
+  // wait for the incoming KV.  Its launches and bytes are still counted.
   cudaError_t e = launch_memmove(dev_w, src_off, dst_off, bytes, impl_of(cfg, bytes), s_weights, &nl);
   AEG_REQUIRE(e == cudaSuccess, AEG_ERR_CUDA, "relocate launch failed: %s", cudaGetErrorString(e));
-  if (timing) {
-    CUDA_TRY(cudaEventRecord(tb, s_weights));
-    pending_timing.push_back({3, ta, tb});
-  }
   kstats[3].launches += nl;
   kstats[3].bytes += 2 * bytes;
   record(x, 0, s_weights);
