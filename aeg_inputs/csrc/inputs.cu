@@ -235,31 +235,6 @@ int aegin_copy_chunks(void* dst_base, const uint64_t* dst_off, const void* src_b
   return 0;
 }
 
-// The same chunks through the CUDA 12.8+ batched-memcpy API (cudaMemcpyBatchAsync, copy engines
-// only): the strongest library baseline for a paged swap without kernels.  Batches of <= 8192
-// copies per call, stream-ordered source access.
-int aegin_copy_chunks_batch(void* dst_base, const uint64_t* dst_off, const void* src_base, const uint64_t* src_off,
-                            uint64_t n, uint64_t chunk, void* stream) {
-  const uint64_t B = 8192;
-  std::vector<void*> d(B), s(B);
-  std::vector<size_t> z(B, size_t(chunk));
-  cudaMemcpyAttributes attr{};
-  attr.srcAccessOrder = cudaMemcpySrcAccessOrderStream;
-  size_t idx0 = 0;
-  for (uint64_t a = 0; a < n; a += B) {
-    const uint64_t m = (n - a < B) ? n - a : B;
-    for (uint64_t i = 0; i < m; ++i) {
-      d[i] = static_cast<char*>(dst_base) + dst_off[a + i];
-      s[i] = const_cast<char*>(static_cast<const char*>(src_base)) + src_off[a + i];
-    }
-    size_t fail = 0;
-    cudaError_t e = cudaMemcpyBatchAsync(d.data(), s.data(), z.data(), size_t(m), &attr, &idx0, 1, &fail,
-                                         static_cast<cudaStream_t>(stream));
-    if (e != cudaSuccess) return int(e);
-  }
-  return 0;
-}
-
 // Load every kernel of this library now (no lazy module load later, which would wait for a
 // running gate kernel and deadlock a race test).
 int aegin_preload(void) {

@@ -34,7 +34,6 @@ def lib():
             "aegin_host_fill": [P, U64, U64, U64, C.c_int],
             "aegin_host_fill_2d": [P, U64, U64, U64, U64, U64, C.c_int],
             "aegin_copy_chunks": [P, PU64, P, PU64, U64, U64, P],
-            "aegin_copy_chunks_batch": [P, PU64, P, PU64, U64, U64, P],
             "aegin_stamp": [P, P],
         }
         for k, a in sig.items():
@@ -137,13 +136,6 @@ def copy_chunks(dst_base: int, dst_offs, src_base: int, src_offs, chunk: int, st
     d, s_ = _u64(dst_offs), _u64(src_offs)
     _ck(lib().aegin_copy_chunks(P(dst_base), d.ctypes.data_as(PU64), P(src_base), s_.ctypes.data_as(PU64), d.size,
                                 chunk, P(stream)))
-
-
-def copy_chunks_batch(dst_base: int, dst_offs, src_base: int, src_offs, chunk: int, stream: int = 0):
-    """The same chunks through cudaMemcpyBatchAsync (batches of <= 8192 copies; batched-API baseline)."""
-    d, s_ = _u64(dst_offs), _u64(src_offs)
-    _ck(lib().aegin_copy_chunks_batch(P(dst_base), d.ctypes.data_as(PU64), P(src_base), s_.ctypes.data_as(PU64),
-                                      d.size, chunk, P(stream)))
 
 
 def stamp(dev_u64_ptr: int, stream: int = 0):

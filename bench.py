@@ -480,9 +480,8 @@ class SwapBench:
 def chunk_memcpy_baseline(aeg, torch, ctx, sht, src_blocks, reps=2):
     """The per-block memcpy the paper's swap amounts to for paged KV ("memcpy(async)"
     Fig. 10; vLLM-style swap_blocks): one cudaMemcpyAsync per (block, layer) chunk, device blocks ->
-    host blocks, then host -> fresh device blocks, on one stream (copy engines only); and the same
-    chunks through the batched-memcpy API (cudaMemcpyBatchAsync, `batch_api_*`).  Same blocks and
-    placement as the library's swap; timed with CUDA events.  Returns GB/s per direction."""
+    host blocks, then host -> fresh device blocks, on one stream (copy engines only).  Same blocks
+    and placement as the library's swap; timed with CUDA events.  Returns GB/s per direction."""
     from aeg_inputs import dev as D
     sh = aeg.KVShape.of(sht)
     n = len(src_blocks)
@@ -493,17 +492,16 @@ def chunk_memcpy_baseline(aeg, torch, ctx, sht, src_blocks, reps=2):
     so, ho, no = (chunk_offsets(ctx, p, sht, b) for p, b in ((0, src_blocks), (1, hc), (0, nd)))
     s = new_stream(torch)
     out = {}
-    for fn, pre in ((D.copy_chunks, ""), (D.copy_chunks_batch, "batch_api_")):
-        for name, args in (("d2h", (hbase, ho, dbase, so)), ("h2d", (dbase, no, hbase, ho))):
-            ts = []
-            for _ in range(reps):
-                e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-                e0.record(s)
-                fn(*args, sh.chunk_bytes(), s.cuda_stream)
-                e1.record(s)
-                e1.synchronize()
-                ts.append(e0.elapsed_time(e1))
-            out[pre + name + "_GBps"] = round(n * sh.block_bytes() / (min(ts) * 1e6), 2)
+    for name, args in (("d2h", (hbase, ho, dbase, so)), ("h2d", (dbase, no, hbase, ho))):
+        ts = []
+        for _ in range(reps):
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record(s)
+            D.copy_chunks(*args, sh.chunk_bytes(), s.cuda_stream)
+            e1.record(s)
+            e1.synchronize()
+            ts.append(e0.elapsed_time(e1))
+        out[name + "_GBps"] = round(n * sh.block_bytes() / (min(ts) * 1e6), 2)
     out["memcpy_calls_per_direction"] = int(so.size)
     out["chunk_bytes"] = sh.chunk_bytes()
     ctx.kv_free(aeg.POOL_HOST, hc)
@@ -948,17 +946,15 @@ def migrate_leg(aeg, torch, kernel, n_req=16, src_layout=None, dst_layout=None):
     doffs = chunk_offsets(b, 0, sht, dc)
     bad, _ = D.verify_chunks(bbase, doffs, keys, sh.chunk_bytes(), seed)
     # baseline on the same blocks: one cudaMemcpyAsync (copy engine, D2D) per (block, layer) chunk
-    # and the same chunks through cudaMemcpyBatchAsync: the copy-engine route with zero SMs
     s = new_stream(torch)
-    bt, bb = [], []
-    for fn, acc in ((D.copy_chunks, bt), (D.copy_chunks_batch, bb)):
-        for _ in range(2):
-            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-            e0.record(s)
-            fn(bbase, doffs, abase, offs, sh.chunk_bytes(), s.cuda_stream)
-            e1.record(s)
-            e1.synchronize()
-            acc.append(e0.elapsed_time(e1))
+    bt = []
+    for _ in range(2):
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(s)
+        D.copy_chunks(bbase, doffs, abase, offs, sh.chunk_bytes(), s.cuda_stream)
+        e1.record(s)
+        e1.synchronize()
+        bt.append(e0.elapsed_time(e1))
     a.shutdown()
     b.shutdown()
     payload = n * sh.block_bytes()
@@ -970,7 +966,6 @@ def migrate_leg(aeg, torch, kernel, n_req=16, src_layout=None, dst_layout=None):
             "kernel_ms_per_xfer": round(kms, 3), "bit_exact": bad == 0,
             "GBps_payload_by_ctas": sweep,
             "per_chunk_memcpy_baseline_GBps_payload": round(payload / (min(bt) * 1e6), 1),
-            "batch_api_ce_baseline_GBps_payload": round(payload / (min(bb) * 1e6), 1),
             "per_chunk_memcpy_calls": int(len(offs))}
 
 
@@ -1078,9 +1073,9 @@ def migrate_leg_dist(aeg, torch, dist, kernel, n_req=16):
         keys = [gi.kv_key(1, sender, i, l) for i in range(n) for l in range(sh.num_layers)]
         bad, _ = D.verify_chunks(base, offs, keys, sh.chunk_bytes(), seed)
     bad = dist.sum(bad)
-    # CE-vs-SM: the same chunks paged -> paged through cudaMemcpyBatchAsync (copy
-    # engines, zero SMs) into the partner's pool mapped here (aeg_peer_region); decode ranks send
-    # their chunk offsets.  Max-over-ranks device time of one round, all pairs at once.
+    # CE-vs-SM: the same chunks paged -> paged, one cudaMemcpyAsync per (block,
+    # layer) chunk (copy engines, zero SMs) into the partner's pool mapped here (aeg_peer_region);
+    # decode ranks send their chunk offsets.  Max-over-ranks device time of one round, all pairs.
     doffs_by_rank = PD.exchange(None if prefill else chunk_offsets(ctx, 0, sht, dst).tolist())
     ce_err = []
 
@@ -1094,7 +1089,7 @@ def migrate_leg_dist(aeg, torch, dist, kernel, n_req=16):
                 s = new_stream(torch)
                 e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
                 e0.record(s)
-                D.copy_chunks_batch(pbase, np.asarray(doffs_by_rank[d], np.uint64), base, offs, sh.chunk_bytes(),
+                D.copy_chunks(pbase, np.asarray(doffs_by_rank[d], np.uint64), base, offs, sh.chunk_bytes(),
                                     s.cuda_stream)
                 e1.record(s)
                 e1.synchronize()
@@ -1107,7 +1102,7 @@ def migrate_leg_dist(aeg, torch, dist, kernel, n_req=16):
     failed = dist.sum(1 if ce_err else 0)
     ce = ({"error": ce_err[0] if ce_err else "failed on another rank"} if failed or ce_ms <= 0 else
           {"GBps_aggregate": round(len(pairs) * n * sh.block_bytes() / (ce_ms * 1e6), 1),
-           "what": "cudaMemcpyBatchAsync of the same (block, layer) chunks, copy engines only"})
+           "what": "one cudaMemcpyAsync per (block, layer) chunk into the peer pool, copy engines only"})
     # SURVEY §8(d) C3 for N >= 4: all-to-all, every prefill rank -> every decode rank, round-robin
     a2a = None
     if world >= 4:
@@ -1122,7 +1117,7 @@ def migrate_leg_dist(aeg, torch, dist, kernel, n_req=16):
     ms = statistics.median(times)
     payload = len(pairs) * n * sh.block_bytes()
     return {"workload": f"configs[2] Llama-2-13B hand-off, {n_req} requests per pair, pairs {pairs}",
-            "nccl_sendrecv_contiguous_baseline": nccl, "batch_api_ce_route": ce,
+            "nccl_sendrecv_contiguous_baseline": nccl, "per_chunk_ce_route": ce,
             "payload_bytes": payload, "ms": round(ms, 3), "GBps_aggregate": round(payload / (ms * 1e6), 1),
             "GBps_per_pair": round(payload / len(pairs) / (ms * 1e6), 1), "peak_per_direction_nominal": NVLINK_NOMINAL,
             "frac_of_nvlink_nominal_per_pair": round(payload / len(pairs) / (ms * 1e6) / NVLINK_NOMINAL, 3),
@@ -1641,7 +1636,7 @@ def run_reference(args):
     value = 2 * sample * bb * args.steps / t / 1e9
     out = {"impl": "reference", "metric": METRIC, "value": round(value, 3), "unit": "GB/s", "n_gpus": args.gpus,
            "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(1e3 * t / args.steps, 1),
-           "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "u8", "data": "synthetic",
+           "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "bf16", "data": "synthetic",
            "config": {"workload": "configs[1] Qwen-7B 64-request swap round trip (bounded sample: "
                                   f"{sample} of {sum(blocks)} blocks per step)", "requests": args.requests},
            "cpu_baseline": {"value": round(value, 3), "unit": "GB/s", "cores": 1, "kind": "oracle",
@@ -1814,7 +1809,7 @@ def run_ours(args):
             "metric": METRIC, "value": round(value, 2), "unit": "GB/s", "n_gpus": world, "steps": args.steps,
             "warmup": args.warmup, "ms_per_step": round(ms_step, 2),
             "step_ms_p10_p50_p90": [pct(0.1), pct(0.5), pct(0.9)], "higher_is_better": True, "scaling": "weak",
-            "vs_baseline": None, "dtype": "u8", "data": "synthetic",
+            "vs_baseline": None, "dtype": "bf16", "data": "synthetic",
             "config": {"workload": "configs[1]: Qwen-7B-shaped KV (32 layers, 32 KV heads, d=128, bf16, 16-token "
                                    f"blocks), {n_req}-request decode batch swapped out and back in per step",
                        "requests": n_req, "tokens": int(sum(sb.lens)), "blocks": sb.n,

@@ -57,7 +57,8 @@ def _build_lib(name: str, srcs: list[str], incs: list[str], headers: list[str], 
             f.result()
     if force or jobs or _needs(out, objs):
         tmp = out + ".tmp"
-        _run([NVCC] + ARCH + ["-shared", "-o", tmp] + objs + ["-lpthread"], log)
+        _run([NVCC] + ARCH + ["-shared", "-cudart", "shared", "-Xlinker", f"-rpath,{CUDA}/lib64", "-o", tmp]
+             + objs + ["-lpthread"], log)
         os.replace(tmp, out)
     return out
 
