@@ -188,7 +188,8 @@ int aeg_kv_free(aeg_ctx ctx, int32_t pool, const aeg_block* blocks, int32_t n);
  * in-flight transfer.  Returns AEG_OK. */
 int aeg_reclaim(aeg_ctx ctx, int blocking);
 
-/* Pool statistics (fragmentation = unused / allocated, from the fields). */
+/* Pool statistics.  Fig. 16's fragmentation, "the ratio of unused memory to peak allocated memory"
+ * (PAPER.md:2030-2033), is (assigned_bytes - used_bytes) / peak_assigned_bytes. */
 int aeg_stats(aeg_ctx ctx, int32_t pool, aeg_pool_stats* out);
 
 /* Decode a handle.  Any output pointer may be NULL. */

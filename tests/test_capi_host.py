@@ -117,6 +117,10 @@ class Pair:
         assert got == per
         used = sum(v[1] * sh.block_bytes() for sh, v in per.items())
         assert s.used_bytes == used
+        # Fig. 16's fragmentation (unused / peak allocated) from the library's own fields
+        assert s.peak_assigned_bytes == self.o.peak_assigned
+        frag = 0.0 if s.peak_assigned_bytes == 0 else (s.assigned_bytes - s.used_bytes) / s.peak_assigned_bytes
+        assert frag == pytest.approx(self.o.fragmentation())
 
     def run(self, ops):
         for op in ops:

@@ -202,9 +202,35 @@ def test_errors_and_all_or_nothing():
     assert e.value.code in (STATE, INVALID)
 
 
-def test_fragmentation_metric():
+def test_fragmentation_metric_hand_trace():
+    """Fig. 16's metric, "unused memory to peak allocated memory", on a
+    4-step trace whose values are worked out by hand from that definition (slab 256 B; A blocks
+    128 B, two per slab; Bsh blocks 192 B, one per slab)."""
     p = SlabPool(4 * SLAB, SLAB)
-    p.alloc(A, 1)                      # one 256 B slab, 128 B used
+    a = p.alloc(A, 1)        # assigned 256, used 128, peak 256 -> 128/256
     assert p.fragmentation() == pytest.approx(0.5)
-    p.alloc(Bsh, 1)                    # + one slab, 192 B used -> unused 192 of 512
-    assert p.fragmentation() == pytest.approx((512 - 128 - 192) / 512)
+    p.alloc(Bsh, 1)          # assigned 512, used 320, peak 512 -> 192/512
+    assert p.fragmentation() == pytest.approx(0.375)
+    p.free(a)                # A's slab reclaimed: assigned 256, used 192, peak stays 512 -> 64/512
+    assert p.fragmentation() == pytest.approx(0.125)
+    assert p.unused_over_assigned() == pytest.approx(0.25)       # the current-denominator figure
+    p.alloc(A, 2)            # slab 0 back for A, full: assigned 512, used 448, peak 512 -> 64/512
+    assert p.fragmentation() == pytest.approx(0.125)
+    # per shape: A peaked at 256 B (one slab) and now fills it; Bsh peaked at 256 B, uses 192
+    assert p.fragmentation(A) == pytest.approx(0.0)
+    assert p.fragmentation(Bsh) == pytest.approx(64 / 256)
+
+
+def test_fragmentation_empty_pool_and_slab_tail():
+    p = SlabPool(4 * SLAB, SLAB)
+    assert p.fragmentation() == 0.0
+    C3 = KVShape(L=1, H=1, D=5, s=2, B=8)     # chunk = block = 2*1*5*2*8 = 160 B -> 1 per slab, 96 B tail
+    c = p.alloc(C3, 1)
+    assert p.fragmentation() == pytest.approx(96 / 256)
+    b = p.alloc(Bsh, 2)      # assigned 768 (peak), used 160 + 384
+    assert p.fragmentation() == pytest.approx((768 - 544) / 768)
+    p.free(b)
+    p.free(c)                # everything reclaimed: assigned 0, peak 768
+    assert p.fragmentation() == 0.0
+    p.alloc(A, 1)            # assigned 256, used 128; the peak is still 768 -> 128/768
+    assert p.fragmentation() == pytest.approx(128 / 768)

@@ -87,3 +87,22 @@ def test_region_exhausted():
     tens = [tensor(d["rows"], d["cols"], k) for k, d in enumerate(descs)]
     with pytest.raises(W.WeightError):
         W.stage(tens, descs, 0, 1, region_bytes=1 << 16)
+
+
+def test_region_exact_fit_and_one_byte_over():
+    """Reading 17's bump layout: the region must hold [base, off_last + size_last); an exact fit
+    stages, one byte less raises (pins the boundary of the exhaustion check)."""
+    descs = gi.model_tensors("tiny")
+    tens = [tensor(d["rows"], d["cols"], k) for k, d in enumerate(descs)]
+    sizes = [W.shard(t.reshape(d["rows"], d["cols"], 2), d["split"], d["groups"], 0, 1).size
+             for t, d in zip(tens, descs)]
+    base = 512
+    p, last = base, base
+    for n in sizes:                  # worked out independently of bump_offsets: align each start
+        last = p
+        p = (p + n + 255) // 256 * 256
+    need = last + sizes[-1]
+    img, offs, _ = W.stage(tens, descs, 0, 1, region_bytes=need, base=base)
+    assert img.size == need and offs[-1] == last
+    with pytest.raises(W.WeightError):
+        W.stage(tens, descs, 0, 1, region_bytes=need - 1, base=base)

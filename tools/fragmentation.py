@@ -8,7 +8,8 @@ allocator (host-only context: the same C++ code as the GPU build, no CUDA) for s
 
 Trace recipe: per model a Poisson request stream (popularity skewed 1/rank), prompt +
 output lengths lognormal (ShareGPT-like means ~ 600 / 300 tokens), a request holds ceil(T/16) blocks
-for an exponential residence time; load set so the cache runs at ~60-80% occupancy.
+for an exponential residence time; load set (Little's law) for a target mean occupancy of the pool (default 50% and 70%); the
+achieved occupancy and any OOMs are reported next to each fragmentation value.
 
     python tools/fragmentation.py [--events N] [--out profiles/fragmentation.json]
 """
@@ -31,16 +32,16 @@ SHAPES = [("S0 Qwen-7B", 32, 32, 128), ("S1 InternLM2.5-7B", 32, 8, 128), ("S2 L
           ("S3 Qwen-72B/TP4", 80, 16, 128), ("S4 Qwen-1.8B", 24, 16, 128), ("S5 Yi-9B", 48, 4, 128)]
 
 
-def trace(n_events: int, pool_bytes: int, seed: int = 3000):
+def trace(n_events: int, pool_bytes: int, seed: int = 3000, occupancy: float = 0.5):
     """Seeded list of (time, kind, model, blocks) events; kind 'a' alloc, 'f' free of that request."""
     g = np.random.Generator(np.random.PCG64(seed))
     pop = 1.0 / np.arange(1, len(SHAPES) + 1)
     pop /= pop.sum()
     block = [L * 2 * H * D * 2 * 16 for _, L, H, D in SHAPES]
-    mean_tokens = 900.0
+    mean_tokens = np.exp(np.log(600) + 0.32) + np.exp(np.log(300) + 0.32)   # E[lognormal] = e^(mu + s^2/2)
     mean_bytes = sum(p * b * mean_tokens / 16 for p, b in zip(pop, block))
     hold = 30.0                                       # mean residence (s)
-    rate = 0.6 * pool_bytes / (mean_bytes * hold)     # Little's law: ~60% occupancy
+    rate = occupancy * pool_bytes / (mean_bytes * hold)   # Little's law: mean used bytes
     t, ev, heap, rid = 0.0, [], [], 0
     while len(ev) < n_events:
         t += g.exponential(1.0 / rate)
@@ -79,7 +80,7 @@ def run(ev, pool_bytes: int, slab_bytes: int):
             if r in live:
                 ctx.kv_free(aeg.POOL_HOST, live.pop(r))
         s = ctx.stats(aeg.POOL_HOST)
-        samples.append((s.assigned_bytes, s.used_bytes))
+        samples.append((s.assigned_bytes, s.used_bytes, s.peak_assigned_bytes))
         if s.assigned_bytes > peak[0]:
             per = {}
             for i in range(s.n_shapes):
@@ -91,28 +92,37 @@ def run(ev, pool_bytes: int, slab_bytes: int):
             peak = (s.assigned_bytes, s.used_bytes, per)
     ctx.shutdown()
     a = np.array(samples, dtype=np.float64)
-    busy = a[:, 0] > 0
-    frac = (a[busy, 0] - a[busy, 1]) / a[busy, 0]
+    a = a[len(a) // 10:]                       # drop the fill-up transient (first 10% of events)
+    frag = (a[:, 0] - a[:, 1]) / a[:, 2]       # Fig. 16: unused / peak allocated, at every event
+    occ = a[:, 1] / pool_bytes
     return {"slab_GiB": slab_bytes / GIB, "events": len(ev), "oom_allocs": oom,
+            "occupancy_used_over_pool_mean": round(float(occ.mean()), 4),
+            "occupancy_used_over_pool_max": round(float(occ.max()), 4),
+            "frag_unused_over_peak_allocated_mean": round(float(frag.mean()), 4),
+            "frag_unused_over_peak_allocated_p90": round(float(np.quantile(frag, 0.9)), 4),
             "frag_at_peak_allocated": round(1 - peak[1] / peak[0], 4) if peak[0] else None,
-            "unused_over_peak_allocated_mean": round(float(((a[:, 0] - a[:, 1]) / peak[0]).mean()), 4),
-            "frag_time_mean": round(float(frac.mean()), 4), "frag_time_p90": round(float(np.quantile(frac, 0.9)), 4),
             "peak_allocated_GiB": round(peak[0] / GIB, 1),
-            "per_shape_at_peak": {k: round(v, 4) for k, v in (peak[2] or {}).items()}}
+            "per_shape_unused_over_assigned_at_peak": {k: round(v, 4) for k, v in (peak[2] or {}).items()}}
 
 
 def main():
     p = argparse.ArgumentParser()
     p.add_argument("--events", type=int, default=60000)
     p.add_argument("--pool-gib", type=int, default=320)     # "Unified CPU KV Cache (320 GB)", Fig. 9
+    p.add_argument("--occupancy", default="0.5,0.7")
     p.add_argument("--slabs", default="0.25,0.5,1,2,4")
     p.add_argument("--out", default=os.path.join(ROOT, "profiles", "fragmentation.json"))
     a = p.parse_args()
     from paper_conf_sosp_xiang0qyzyzl0025_b200 import build
     build.build()
     pool = a.pool_gib * GIB
-    ev = trace(a.events, pool)
-    res = [run(ev, pool, int(float(s) * GIB)) for s in a.slabs.split(",")]
+    res = []
+    for occ in (float(x) for x in a.occupancy.split(",")):
+        ev = trace(a.events, pool, occupancy=occ)
+        for s in a.slabs.split(","):
+            r = run(ev, pool, int(float(s) * GIB))
+            r["target_mean_occupancy"] = occ
+            res.append(r)
     out = {"what": "N3 fragmentation of the unified CPU KV cache (slab allocator of libaegkv, host-only)",
            "paper": "overall < 20% (PAPER.md:2068-2070, Fig. 16)", "pool_GiB": a.pool_gib, "results": res}
     os.makedirs(os.path.dirname(a.out), exist_ok=True)

@@ -25,6 +25,10 @@ MUTANTS = [
     ("oracle/weights.py", "p = align_up(p + n)", "p = p + n"),
     ("oracle/memmove.py", "out[dst:dst + n] = tmp", "out[dst:dst + n] = tmp[::-1]"),
     ("oracle/memmove.py", "tmp = buf[src:src + n].copy()", "tmp = buf[dst:dst + n].copy()"),
+    ("oracle/weights.py", "if offs and offs[-1] + shards[-1].size > region_bytes:", "if offs and offs[-1] > region_bytes:"),
+    ("oracle/weights.py", "if offs and offs[-1] + shards[-1].size > region_bytes:", "if offs and offs[-1] + shards[-1].size >= region_bytes:"),
+    ("oracle/slab.py", "return 0.0 if peak == 0 else (assigned - used) / peak", "return 0.0 if assigned == 0 else (assigned - used) / assigned"),
+    ("oracle/slab.py", "self.peak_assigned = max(self.peak_assigned, sum(v[0] for v in per.values()) * self.slab_bytes)", "self.peak_assigned = sum(v[0] for v in per.values()) * self.slab_bytes"),
     ("oracle/rules.py", "pending.setdefault(e[1], set()).add(c)", "pass"),
     ("oracle/rules.py", "captured[e[2]] = tail.get(e[1])", "captured[e[2]] = len(ops) - 1 if ops else None"),
 ]
