@@ -332,7 +332,11 @@ int aeg_import_peer(aeg_ctx ctx, int32_t peer, const void* buf, uint64_t len);
  * wait on them; aeg_xfer_import turns such a blob into a local transfer id of the importer.  A
  * swap-out whose D2H ran in pieces (aeg_config.dma_piece_mib) also exports its per-(layer, piece)
  * events, piece table and written host handles, so a peer's aeg_kv_swap_in_from(after = it) waits
- * per piece (sub-layer rule ❷ across instances).  Call with buf = NULL to get the size. */
+ * per piece (sub-layer rule ❷ across instances).  Call with buf = NULL to get the size.
+ * Lifetime: export before aeg_xfer_release (AEG_ERR_STATE after).  Another process opens the events
+ * by IPC handle and owns those.  A context in the SAME process borrows the exporter's events: the
+ * exporter keeps the transfer (does not recycle its events) until every such import has been
+ * released and reaped, and the exporting context must be shut down after its importers. */
 int aeg_xfer_export(aeg_ctx ctx, aeg_xfer x, void* buf, uint64_t* len);
 int aeg_xfer_import(aeg_ctx ctx, int32_t peer, const void* buf, uint64_t len, aeg_xfer* out);
 

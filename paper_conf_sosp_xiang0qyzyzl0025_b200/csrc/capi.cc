@@ -86,6 +86,7 @@ struct XferBlobHead {
   // n written host handles in transfer order (0 pieces: nothing follows).
   int32_t npiece;
   int32_t n;
+  uint64_t serial;  // exporter's process-wide transfer serial (same-process imports pin it)
 };
 
 uint64_t xfer_blob_bytes(int32_t L, int32_t npiece, int32_t n) {
@@ -572,7 +573,9 @@ int aeg_xfer_export(aeg_ctx ctx, aeg_xfer xid, void* buf, uint64_t* len) {
     }
     AEG_REQUIRE(*len >= need, AEG_ERR_INVALID, "buffer too small");
     set_device(c);
-    XferBlobHead h{kXferMagic, int32_t(getpid()), x->L, x->ipc ? 1 : 0, x->id, np, nb};
+    AEG_REQUIRE(!x->released, AEG_ERR_STATE, "transfer already released");
+    XferBlobHead h{kXferMagic, int32_t(getpid()), x->L, x->ipc ? 1 : 0, x->id, np, nb,
+                   x->serial};
     char* o = static_cast<char*>(buf);
     std::memcpy(o, &h, sizeof h);
     auto put_event = [&](cudaIpcEventHandle_t* hd, cudaEvent_t e) {
@@ -623,6 +626,7 @@ int aeg_xfer_import(aeg_ctx ctx, int32_t peer, const void* buf, uint64_t len, ae
         reinterpret_cast<const cudaIpcEventHandle_t*>(static_cast<const char*>(buf) + sizeof h);
     auto x = std::make_unique<aeg::Xfer>();
     x->id = c.next_xid++;
+    x->serial = aeg::xfer_next_serial();
     x->kind = aeg::X_IMPORTED;
     x->L = h.L;
     x->owns_events = false;
@@ -670,6 +674,10 @@ int aeg_xfer_import(aeg_ctx ctx, int32_t peer, const void* buf, uint64_t len, ae
       x->npiece = h.npiece;
     }
     x->done_recorded = true;
+    if (same) {  // keep the exporter's events alive until this import is reaped
+      x->pinned_serial = h.serial;
+      aeg::xfer_pin_add(h.serial);
+    }
     *out = x->id;
     c.xfers.emplace(x->id, std::move(x));
     return AEG_OK;

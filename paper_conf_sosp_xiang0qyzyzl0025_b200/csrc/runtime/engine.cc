@@ -217,7 +217,10 @@ void Ctx::shutdown() {
   if (host_only) return;
   for (auto& kv : xfers) {
     Xfer* x = kv.second.get();
-    if (!x->owns_events) continue;
+    if (x->pinned_serial) xfer_pin_drop(x->pinned_serial);
+    // still imported by a same-process context (aeg.h: exporters outlive imports): leak its
+    // events rather than destroy events that context may still wait on
+    if (!x->owns_events || xfer_pinned(x->serial)) continue;
     for (cudaEvent_t e : x->ev) cudaEventDestroy(e);
     if (x->done_ev) cudaEventDestroy(x->done_ev);
   }
@@ -342,7 +345,8 @@ void Ctx::housekeeping() {
   // reap released + completed transfers, recycle their events
   for (auto it = xfers.begin(); it != xfers.end();) {
     Xfer* x = it->second.get();
-    if (x->released && x->complete.load()) {
+    if (x->released && x->complete.load() && !xfer_pinned(x->serial)) {
+      if (x->pinned_serial) xfer_pin_drop(x->pinned_serial);
       if (x->owns_events && !host_only) {
         for (cudaEvent_t e : x->ev) give_event(e, x->ipc);
         if (x->done_ev) give_event(x->done_ev, x->ipc);
@@ -375,9 +379,31 @@ cudaEvent_t Ctx::take_event(bool ipc) {
 
 void Ctx::give_event(cudaEvent_t e, bool ipc) { (ipc ? ev_pool_ipc : ev_pool).push_back(e); }
 
+namespace {
+std::mutex g_pin_mu;
+std::unordered_map<uint64_t, int32_t> g_pins;
+std::atomic<uint64_t> g_serial{1};
+}  // namespace
+
+uint64_t xfer_next_serial() { return g_serial.fetch_add(1); }
+void xfer_pin_add(uint64_t serial) {
+  std::lock_guard<std::mutex> g(g_pin_mu);
+  ++g_pins[serial];
+}
+void xfer_pin_drop(uint64_t serial) {
+  std::lock_guard<std::mutex> g(g_pin_mu);
+  auto it = g_pins.find(serial);
+  if (it != g_pins.end() && --it->second <= 0) g_pins.erase(it);
+}
+bool xfer_pinned(uint64_t serial) {
+  std::lock_guard<std::mutex> g(g_pin_mu);
+  return g_pins.count(serial) != 0;
+}
+
 Xfer* Ctx::new_xfer(int kind, int32_t L, bool ipc) {
   auto x = std::make_unique<Xfer>();
   x->id = next_xid++;
+  x->serial = xfer_next_serial();
   x->kind = kind;
   x->L = L;
   x->ipc = ipc;

@@ -45,6 +45,11 @@ struct Xfer {
   std::atomic<bool> complete{false};
   bool released = false;
   bool owns_events = true;          // imported transfers borrow cached peer events
+  // Same-process imports borrow the exporter's raw events: while a process-wide pin on `serial`
+  // is held (xfer_pin_*) the exporter keeps this transfer and its events; an imported copy holds
+  // the pin on `pinned_serial` until it is reaped or its context shuts down.
+  uint64_t serial = 0;
+  uint64_t pinned_serial = 0;
   bool failed = false;              // enqueue was interrupted by an error (events force-recorded)
   bool debug_done = false;          // host-only synthetic transfers
   uint64_t table_mark = 0;          // table-arena end offset to release on completion
@@ -59,6 +64,12 @@ struct Xfer {
   std::vector<cudaEvent_t> pev;
   std::unordered_map<aeg_block, int32_t> wpos;  // written host block -> its index in the transfer
 };
+
+// Process-wide pins of exported transfers (serial numbers), for same-process imports.
+uint64_t xfer_next_serial();
+void xfer_pin_add(uint64_t serial);
+void xfer_pin_drop(uint64_t serial);
+bool xfer_pinned(uint64_t serial);
 
 // Device staging ring for one direction of KV swaps: a byte ring (slots x slot_bytes) in which
 // segments of any size <= slot_bytes are packed back to back.  Reuse is ordered entirely on the

@@ -118,6 +118,19 @@ std::vector<std::pair<int32_t, int32_t>> pieces_of(const Seg& g, uint64_t chunk,
 
 }  // namespace
 
+// Largest pitch a 2-D copy accepts (cudaDevAttrMaxPitch, 2^31-1 on B200), queried once.  Runs in
+// slabs further apart than this (e.g. whole 1 GiB slabs 0, 2, 4 -> pitch 2 GiB) are not merged.
+static int64_t max_pitch() {
+  static const int64_t v = [] {
+    int dev = 0, mp = 0;
+    if (cudaGetDevice(&dev) != cudaSuccess || cudaDeviceGetAttribute(&mp, cudaDevAttrMaxPitch, dev) != cudaSuccess ||
+        mp <= 0)
+      return int64_t(INT32_MAX);
+    return int64_t(mp);
+  }();
+  return v;
+}
+
 // Copy-engine DMAs between a staging slot and the host blocks of segment g (layer-major staging
 // image inside the slot).  dir = cudaMemcpyDeviceToHost (swap-out) or HostToDevice (swap-in).
 static void host_dmas(const SlabPool& hp, char* hbase, const Shape& sh, const std::vector<Run>& runs, const Seg& g,
@@ -150,7 +163,7 @@ static void host_dmas(const SlabPool& hp, char* hbase, const Shape& sh, const st
         char* cur = host_of(r, r.i0);
         const int64_t p = cur - prev;
         if (e == q + 1) pitch = p;
-        if (p != pitch || p < int64_t(m) * int64_t(Cl)) break;
+        if (p != pitch || p < int64_t(m) * int64_t(Cl) || p > max_pitch()) break;
         prev = cur;
         ++e;
       }
@@ -182,11 +195,15 @@ static void host_dmas(const SlabPool& hp, char* hbase, const Shape& sh, const st
     if (hp.layout == AEG_LAYER_MAJOR) {
       // the run is contiguous within each layer: one 1-D copy, or one 2-D copy over the layers
       const uint64_t w = uint64_t(m) * Cl;
-      if (nl == 1) {
-        if (dir == cudaMemcpyDeviceToHost)
-          CUDA_TRY(cudaMemcpyAsync(host0, st0, w, dir, s));
-        else
-          CUDA_TRY(cudaMemcpyAsync(st0, host0, w, dir, s));
+      if (nl == 1 || int64_t(hstride) > max_pitch()) {
+        for (int32_t t = 0; t < nl; ++t) {
+          char* h = host0 + uint64_t(t) * hstride;
+          char* st = st0 + uint64_t(t) * st_pitch;
+          if (dir == cudaMemcpyDeviceToHost)
+            CUDA_TRY(cudaMemcpyAsync(h, st, w, dir, s));
+          else
+            CUDA_TRY(cudaMemcpyAsync(st, h, w, dir, s));
+        }
       } else if (dir == cudaMemcpyDeviceToHost) {
         CUDA_TRY(cudaMemcpy2DAsync(host0, hstride, st0, st_pitch, w, nl, dir, s));
       } else {
@@ -390,11 +407,14 @@ uint64_t Ctx::swap_in_from(const Shape& sh, int32_t peer, const aeg_block* host,
     }
     rdeps.swap(rest);
   }
+  Xfer* after_x = nullptr;  // `after` waited per piece: a piece none of whose blocks it wrote still
+                            // waits for its layer to land (aeg.h: layer l waits on layer l of after)
   if (after) {  // rule ❷ across instances (Fig. 10 ③): per piece if the peer exported pieces
     auto it = xfers.find(after);
-    if (it != xfers.end() && piecewise(it->second.get(), sh.L))
-      pdeps.push_back(it->second.get());
-    else
+    if (it != xfers.end() && piecewise(it->second.get(), sh.L)) {
+      after_x = it->second.get();
+      if (std::find(pdeps.begin(), pdeps.end(), after_x) == pdeps.end()) pdeps.push_back(after_x);
+    } else
       rdeps.push_back(after);
   }
   rdeps = uniq(rdeps);
@@ -428,6 +448,7 @@ uint64_t Ctx::swap_in_from(const Shape& sh, int32_t peer, const aeg_block* host,
                                       w->piece_lo.begin()) - 1;
             hi = std::max(hi, p);
           }
+          if (hi < 0 && w == after_x) hi = w->npiece - 1;  // its last piece of the layer = the layer
           if (hi >= 0) need.push_back({w, hi});
         }
         pneed.push_back(std::move(need));

@@ -97,6 +97,46 @@ def test_same_process_peer_migrate_and_imported_events():
         b.shutdown()
 
 
+def test_same_process_import_pins_the_exporters_events():
+    """a same-process import borrows the exporter's raw events.  After the exporter
+    releases and reaps its transfer, a new gate-held transfer of the exporter must NOT re-record
+    those events (they stay pinned until the import is reaped): the importer still sees every
+    layer complete."""
+    require_gpu()
+    import torch
+    from aeg_inputs import dev as D
+    a, A = make(aeg.LAYER_MAJOR)
+    b, B = make(aeg.BLOCK_MAJOR)
+    try:
+        sc, so = A.alloc(SH, 20)
+        dc, do = A.alloc(SH, 20)
+        x = a.kv_migrate(SH.as_tuple(), sc, -1, dc)
+        a.layer_ready(x, -1, aeg.READY_BLOCK)
+        xi = b.xfer_import(0, a.xfer_export(x))
+        a.xfer_release(x)
+        with pytest.raises(aeg.AegError):
+            a.xfer_export(x)                    # released: no more exports
+        a.reclaim(True)                         # the exporter reaps what it may
+        s = torch.cuda.Stream()
+        gate = D.Gate()
+        gate.close_on(s.cuda_stream)
+        a.stream_fence(s.cuda_stream)
+        ys = [a.kv_migrate(SH.as_tuple(), dc, -1, sc) for _ in range(2)]   # would take recycled events
+        assert not a.layer_ready(ys[0], 0, aeg.READY_QUERY)
+        for l in range(SH.L):
+            assert b.layer_ready(xi, l, aeg.READY_QUERY), f"imported layer {l} re-armed by the exporter"
+        assert b.layer_ready(xi, -1, aeg.READY_QUERY)
+        gate.open()
+        for y in ys:
+            a.layer_ready(y, -1, aeg.READY_BLOCK)
+        b.xfer_release(xi)
+        b.reclaim(True)                         # import reaped: the pin is dropped
+        a.reclaim(True)
+    finally:
+        b.shutdown()
+        a.shutdown()
+
+
 def _decode_side(conn):
     """Child process: the decode instance.  Allocates destination blocks, exports its pool, waits on
     the imported per-layer events, then reports its image."""
