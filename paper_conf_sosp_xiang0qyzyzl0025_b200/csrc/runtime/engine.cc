@@ -257,6 +257,10 @@ char* Ring::acquire(uint64_t size, cudaStream_t producer, cudaEvent_t* full, cud
                    std::vector<cudaEvent_t>* waited) {
   AEG_REQUIRE(size > 0 && size <= slot_bytes, AEG_ERR_INVALID, "staging segment of %llu bytes exceeds a slot",
               (unsigned long long)size);
+  // segments start on 16 KiB boundaries (the trace's ring granule, swap.cc ring_cells): two
+  // segments never share a granule, so ring reuse is exactly what the rule checker sees
+  constexpr uint64_t kRingAlign = 16u << 10;
+  head += (kRingAlign - (head % bytes) % kRingAlign) % kRingAlign;
   const uint64_t pos = head % bytes;
   if (pos + size > bytes) head += bytes - pos;  // never wrap inside a segment
   const uint64_t start = head, end = head + size;

@@ -35,7 +35,7 @@ MODELS3 = [
     ("llama-7b", KVShape(32, 4, 64, 2, 16), dict(h=128, L=32, ff=384, V=2048, arch="llama"), 11),
     ("yi-9b", KVShape(48, 1, 128, 2, 16), dict(h=128, L=48, ff=256, V=3072, arch="llama"), 15),
 ]
-WPOISON = gi.poison_key(gi.TAG_NEVER, 7)
+WPOISON = gi.poison_key(gi.TAG_NEVER, 8 * 7)
 
 
 def _align(x):
