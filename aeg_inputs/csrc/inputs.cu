@@ -92,9 +92,16 @@ __global__ void consume_chunks(const char* base, const uint64_t* off, uint64_t n
 }
 
 // Deterministic race-test gate: holds its stream until the host writes a nonzero value into the
-// pinned (device-mapped) flag.
+// pinned (device-mapped) flag, or at most 60 s (a test that fails while its gate is closed must not
+// hang the GPU: the streams behind the gate drain and the test reports a data mismatch instead).
 __global__ void gate(const volatile int* flag) {
-  while (*flag == 0) __nanosleep(1000);
+  unsigned long long t0, t;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t0));
+  do {
+    if (*flag != 0) return;
+    __nanosleep(1000);
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+  } while (t - t0 < 60ull * 1000000000ull);
 }
 
 // GPU-wide nanosecond clock, comparable across processes sharing the GPU (cross-process timing of

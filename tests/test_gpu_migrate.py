@@ -294,8 +294,8 @@ def test_two_process_host_route_p_c_d(nblocks):
         a.stream_fence(s.cuda_stream)
         xo = a.kv_swap_out(SH.as_tuple(), sc, hc, flags=aeg.FREE_SRC)                            # ①②
         xob = a.xfer_export(xo)
-        # 32-byte head + (L + 1) 64-byte IPC event handles; pieces add their table and events
-        assert (len(xob) > 32 + (SH.L + 1) * 64) == (nblocks * SH.chunk_bytes() > 4 * MIB)
+        # 40-byte head + (L + 1) 64-byte IPC event handles; pieces add their table and events
+        assert (len(xob) > 40 + (SH.L + 1) * 64) == (nblocks * SH.chunk_bytes() > 4 * MIB)
         parent.send(([int(b) for b in hc], xob))
         xblob, do = recv()
         xd = a.xfer_import(1, xblob)
