@@ -200,6 +200,57 @@ class Clocks:
                 "power_w_max": max(float(r[3]) for r in rows if r[3].replace(".", "").isdigit())}
 
 
+class PcieCounters:
+    """NVML PCIe throughput counters of this GPU (nvmlDeviceGetPcieThroughput: bytes over the link in
+    a 20 ms window, per direction) sampled by a thread while the block runs: hardware-counter
+    evidence for the copy-engine traffic that ncu cannot see.  tx = device -> host (D2H), rx =
+    host -> device (H2D); reported in GB/s (NVML's KB/s / 1e6)."""
+
+    def __init__(self, gpu: int):
+        self.gpu, self.rows, self.err = gpu, [], None
+
+    def __enter__(self):
+        import threading
+        self.stop = threading.Event()
+        try:
+            import pynvml as N
+            N.nvmlInit()
+            self.N, self.h = N, N.nvmlDeviceGetHandleByIndex(self.gpu)
+        except Exception as e:  # noqa: BLE001
+            self.err = f"{type(e).__name__}: {e}"
+            return self
+
+        def run():
+            N = self.N
+            while not self.stop.is_set():
+                try:
+                    tx = N.nvmlDeviceGetPcieThroughput(self.h, N.NVML_PCIE_UTIL_TX_BYTES)
+                    rx = N.nvmlDeviceGetPcieThroughput(self.h, N.NVML_PCIE_UTIL_RX_BYTES)
+                except Exception as e:  # noqa: BLE001
+                    self.err = f"{type(e).__name__}: {e}"
+                    return
+                self.rows.append((tx / 1e6, rx / 1e6))
+        self.t = threading.Thread(target=run, daemon=True)
+        self.t.start()
+        return self
+
+    def __exit__(self, *a):
+        self.stop.set()
+        if hasattr(self, "t"):
+            self.t.join(timeout=5)
+
+    def summary(self):
+        if not self.rows:
+            return {"error": self.err or "no samples"}
+        r = self.rows[1:-1] or self.rows          # drop the windows straddling the region's edges
+        tx = sorted(x[0] for x in r)
+        rx = sorted(x[1] for x in r)
+        med = lambda v: round(v[len(v) // 2], 1)  # noqa: E731
+        return {"tx_d2h_GBps_median": med(tx), "rx_h2d_GBps_median": med(rx),
+                "tx_d2h_GBps_mean": round(sum(tx) / len(tx), 1), "rx_h2d_GBps_mean": round(sum(rx) / len(rx), 1),
+                "samples": len(r), "source": "NVML nvmlDeviceGetPcieThroughput (20 ms windows)"}
+
+
 def peaks():
     p = os.path.join(ROOT, "MEASURED_PEAKS.json")
     if os.path.exists(p):
@@ -455,22 +506,24 @@ class SwapBench:
         for name in ("swap_out", "swap_in"):
             self.ctx.kernel_stats_reset()
             e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-            e0.record(cons)
-            self.ctx.stream_fence(cons.cuda_stream)
-            if name == "swap_out":
-                x = self.ctx.kv_swap_out(self.sht, self.src_c, hc, flags=aeg.FREE_SRC)
-            else:
-                x = self.ctx.kv_swap_in(self.sht, hc, nd, flags=aeg.FREE_SRC)
-            self.ctx.layer_ready(x, -1, aeg.READY_WAIT_STREAM, cons.cuda_stream)
-            e1.record(cons)
-            e1.synchronize()
+            with PcieCounters(torch.cuda.current_device()) as pc:
+                e0.record(cons)
+                self.ctx.stream_fence(cons.cuda_stream)
+                if name == "swap_out":
+                    x = self.ctx.kv_swap_out(self.sht, self.src_c, hc, flags=aeg.FREE_SRC)
+                else:
+                    x = self.ctx.kv_swap_in(self.sht, hc, nd, flags=aeg.FREE_SRC)
+                self.ctx.layer_ready(x, -1, aeg.READY_WAIT_STREAM, cons.cuda_stream)
+                e1.record(cons)
+                e1.synchronize()
             self.ctx.layer_ready(x, -1, aeg.READY_BLOCK)
             self.ctx.xfer_release(x)
             ms = e0.elapsed_time(e1)
             k = self.ctx.kernel_stats(aeg.K_GATHER if name == "swap_out" else aeg.K_SCATTER)
             out[name] = {"GBps": round(self.n * self.sh.block_bytes() / (ms * 1e6), 2), "ms": round(ms, 1),
                          "kernel_GBps": round(k[1] / (k[2] * 1e6), 1) if k[2] else None,
-                         "kernel_launches": k[0], "kernel_ms_total": round(k[2], 2)}
+                         "kernel_launches": k[0], "kernel_ms_total": round(k[2], 2),
+                         "nvml_pcie": pc.summary()}
         self.ops.append((hc, nd))
         self.src_c = nd
         return out
@@ -875,10 +928,19 @@ def switch_leg(aeg, torch, n_switch, kernel, descs, mode="staged", caches=None, 
                    "first_layer_ms_p50": round(statistics.median(x["first_ms"] for x in r), 2),
                    "h2d_bytes": int(r[0]["bytes_h2d"]), "weights_bytes": int(wsize[nm]),
                    "h2d_GBps": round(r[0]["bytes_h2d"] / (statistics.median(lat) * 1e6), 1),
-                   "eq4_weights_ms_at_64GBps": round(wsize[nm] / (PCIE_NOMINAL * BETA) / 1e6, 1),
-                   # N4: Eq. 4 solved for beta on this B200: T = size / (BW * beta)
-                   "eq4_beta_fit": None if mode == "prefetch" else
-                   round(wsize[nm] / (PCIE_NOMINAL * 1e9 * statistics.median(lat) / 1e3), 3)}
+                   # N4: Eq. 4 (garbled) predicted and solved for beta on this B200,
+                   # under both readings: literal T = size / BW * beta, and DESIGN reading 19
+                   # T = size / (BW * beta) (an inefficiency lengthens T); paper beta = 0.625
+                   "eq4_weights_ms_at_64GBps": {
+                       "literal": round(wsize[nm] / PCIE_NOMINAL * BETA / 1e6, 1),
+                       "reading19": round(wsize[nm] / (PCIE_NOMINAL * BETA) / 1e6, 1)},
+                   "eq4_beta_fit": None if mode == "prefetch" else {
+                       "literal": round(PCIE_NOMINAL * 1e9 * statistics.median(lat) / 1e3 / wsize[nm], 3),
+                       "reading19": round(wsize[nm] / (PCIE_NOMINAL * 1e9 * statistics.median(lat) / 1e3), 3),
+                       "reading19_all_h2d_bytes": round(r[0]["bytes_h2d"] / (PCIE_NOMINAL * 1e9 * statistics.median(lat) / 1e3), 3),
+                       "what": "size = the model's weight bytes (Eq. 4's Model Size), T = last-layer-ready "
+                               "latency of the switch, which also carries 1 GiB of KV over the same H2D link; "
+                               "reading19_all_h2d_bytes uses weights + KV bytes (the link's own efficiency)"}}
     how = {"staged": "weights staged through the 2 GiB pinned Stage Buffer by host threads (3.a)",
            "direct": "weights DMA'd straight from the page-locked Model Cache (registered once)",
            "prefetch": "weights prefetched during the previous turn, relocated on-device at the switch (3.b)"}[mode]
@@ -1707,7 +1769,7 @@ def run_ours(args):
         sb.step(torch, cons)
     sb.ctx.kernel_stats_reset()
     dist.barrier()
-    with Clocks(dist.device) as clk:
+    with Clocks(dist.device) as clk, PcieCounters(dist.device) as pcnt:
         e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         marks = [torch.cuda.Event(enable_timing=True) for _ in range(args.steps)]
         e0.record(cons)
@@ -1719,6 +1781,7 @@ def run_ours(args):
     dist.barrier()
     ms_total = dist.max(e0.elapsed_time(e1))
     clocks = clk.summary()
+    pcie_counters = pcnt.summary()
     ms_step = ms_total / args.steps
     per_step = sorted(dist.max(a.elapsed_time(b)) for a, b in zip([e0] + marks[:-1], marks))
     pct = lambda q: round(per_step[min(len(per_step) - 1, int(q * (len(per_step) - 1) + 0.5))], 2)  # noqa: E731
@@ -1866,6 +1929,7 @@ def run_ours(args):
                      "peak_per_direction_nominal": PCIE_NOMINAL,
                      "frac_of_duplex_nominal": round(bytes_step / (ms_step * 1e6) / (2 * PCIE_NOMINAL), 3)},
             "clocks": clocks,
+            "pcie_counters": pcie_counters,
             "gpu_launches": launches_all,
             "consumer_launches": args.steps * sb.L,
         }

@@ -82,9 +82,10 @@ enum {
                                    the node-shared "Unified CPU KV Cache" (Fig. 5) */
 };
 /* kernel selection for gather/scatter/migrate.  AEG_KERNEL_AUTO picks the measured best by chunk
- * size Cl: gather/scatter WARP if Cl <= 4 KiB, LSU if Cl < 32 KiB, BULK otherwise;
- * migrate (paged -> paged, local or peer) WARP if Cl <= 4 KiB, LSU otherwise. */
-enum { AEG_KERNEL_AUTO = 0, AEG_KERNEL_LSU = 1, AEG_KERNEL_BULK = 2, AEG_KERNEL_WARP = 3 };
+ * size Cl (profiles/r02/small_chunk_*.txt): gather/scatter WARP if Cl <= 2 KiB, BULKW
+ * (bulk copies issued by several warps per CTA) if Cl <= 16 KiB, BULK otherwise; migrate (paged ->
+ * paged, local or peer) WARP if Cl <= 4 KiB, LSU otherwise. */
+enum { AEG_KERNEL_AUTO = 0, AEG_KERNEL_LSU = 1, AEG_KERNEL_BULK = 2, AEG_KERNEL_WARP = 3, AEG_KERNEL_BULKW = 4 };
 
 /* ---- structs ---------------------------------------------------------------------------- */
 

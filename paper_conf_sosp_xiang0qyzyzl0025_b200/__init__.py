@@ -26,7 +26,7 @@ READY_QUERY, READY_WAIT_STREAM, READY_BLOCK = 0, 1, 2
 FREE_SRC, NO_DEPS = 1, 2
 SPLIT_REPLICATED, SPLIT_COL, SPLIT_ROW, SPLIT_VOCAB = 0, 1, 2, 3
 CFG_HOST_ONLY, CFG_NO_DAEMON, CFG_TIMING, CFG_SHARED_HOST = 1, 2, 4, 8
-KERNEL_AUTO, KERNEL_LSU, KERNEL_BULK, KERNEL_WARP = 0, 1, 2, 3
+KERNEL_AUTO, KERNEL_LSU, KERNEL_BULK, KERNEL_WARP, KERNEL_BULKW = 0, 1, 2, 3, 4
 K_GATHER, K_SCATTER, K_MIGRATE, K_RELOCATE, K_FETCH = 0, 1, 2, 3, 4
 
 

@@ -223,6 +223,104 @@ __global__ void __launch_bounds__(32) copy_bulk(const CopyArgs a) {
   bulk_wait_all();
 }
 
+// ----------------------------------------------------------------------------------- BULKW
+// Small chunks (<= 16 KiB) through the bulk-copy engine: the single-thread BULK above is issue-bound
+// there (one table load, two 64-bit divisions and two cp.async.bulk per 8 KiB, serialised in one
+// thread).  Here a CTA is kBwWarps independent warps, each with its own ring of whole-chunk stages
+// in shared memory (kBwSmem / kBwWarps bytes).  A warp resolves the pointers of 32 of its items at
+// once, one per lane (one coalesced block-table load), and lane 0 issues the bulk copies with the
+// pointers broadcast by __shfl_sync; the ring refill is the BULK pipeline (mbarrier complete_tx for
+// loads, bulk_group read-completion before a stage is reloaded).
+#ifndef AEG_BW_WARPS  // overridable by tools/small_chunk_probe.cu
+#define AEG_BW_WARPS 4
+#endif
+#ifndef AEG_BW_SMEM_KIB
+#define AEG_BW_SMEM_KIB 192
+#endif
+constexpr int kBwWarps = AEG_BW_WARPS;
+#ifndef AEG_BW_MAX_STAGES
+#define AEG_BW_MAX_STAGES 16
+#endif
+constexpr int kBwMaxStages = AEG_BW_MAX_STAGES;
+constexpr int kBwSmem = AEG_BW_SMEM_KIB * 1024;
+
+template <bool SP, bool DP>
+__global__ void __launch_bounds__(kBwWarps * 32) copy_bulkw(const CopyArgs a, uint32_t piece) {
+  extern __shared__ __align__(128) char smem[];
+  __shared__ __align__(8) uint64_t bar[kBwWarps][kBwMaxStages];
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const uint32_t per_warp = uint32_t(kBwSmem / kBwWarps);
+  const uint32_t stages = min(uint32_t(kBwMaxStages), per_warp / piece);
+  char* ring = smem + uint64_t(warp) * per_warp;
+  uint64_t* wb = bar[warp];
+  const uint64_t ppc = (a.chunk + piece - 1) / piece;
+  const uint64_t items = uint64_t(a.nl) * uint64_t(a.n) * ppc;
+  const uint64_t W = uint64_t(gridDim.x) * kBwWarps;
+  const uint64_t gw = uint64_t(blockIdx.x) * kBwWarps + warp;
+  if (gw >= items) return;  // warp-uniform
+  const uint64_t mine = (items - gw + W - 1) / W;
+  if (lane == 0) {
+    for (uint32_t i = 0; i < stages; ++i) mbar_init(&wb[i], 1);
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  __syncwarp();
+  // lane j of a batch holds the pointers of the warp's item 32 * batch + j
+  auto resolve = [&](uint64_t j, const char*& s, char*& d, uint32_t& nb) {
+    const uint64_t w = gw + j * W;
+    const uint64_t c = w / ppc;
+    const uint64_t off = (w - c * ppc) * piece;
+    item_ptrs<SP, DP>(a, c, s, d);
+    s += off;
+    d += off;
+    const uint64_t rem = a.chunk - off;
+    nb = rem < piece ? uint32_t(rem) : piece;
+  };
+  const char* ls = nullptr;
+  char* sd = nullptr;
+  uint32_t lnb = 0, snb = 0;
+  uint64_t lbatch = ~0ull, sbatch = ~0ull;
+  auto load = [&](uint64_t j, uint32_t st) {
+    if ((j >> 5) != lbatch) {  // warp-uniform: j is the same in every lane
+      lbatch = j >> 5;
+      const uint64_t jj = (lbatch << 5) + lane;
+      char* dd;
+      if (jj < mine) resolve(jj, ls, dd, lnb);
+    }
+    const char* s = reinterpret_cast<const char*>(
+        __shfl_sync(0xffffffffu, reinterpret_cast<unsigned long long>(ls), int(j & 31)));
+    const uint32_t nb = __shfl_sync(0xffffffffu, lnb, int(j & 31));
+    if (lane == 0) bulk_load(ring + uint64_t(st) * piece, s, nb, &wb[st]);
+  };
+  auto store = [&](uint64_t j, uint32_t st) {
+    if ((j >> 5) != sbatch) {
+      sbatch = j >> 5;
+      const uint64_t jj = (sbatch << 5) + lane;
+      const char* ss;
+      if (jj < mine) resolve(jj, ss, sd, snb);
+    }
+    char* d = reinterpret_cast<char*>(__shfl_sync(0xffffffffu, reinterpret_cast<unsigned long long>(sd), int(j & 31)));
+    const uint32_t nb = __shfl_sync(0xffffffffu, snb, int(j & 31));
+    if (lane == 0) bulk_store(d, ring + uint64_t(st) * piece, nb);
+  };
+  for (uint64_t j = 0; j < mine && j < stages; ++j) load(j, uint32_t(j));
+  uint32_t st = 0, phase = 0, prev = stages - 1;
+  for (uint64_t k = 0; k < mine; ++k) {
+    if (lane == 0) mbar_wait(&wb[st], phase);
+    __syncwarp();
+    store(k, st);
+    if (k >= 1 && k - 1 + stages < mine) {
+      if (lane == 0) bulk_wait_read<1>();  // the store of item k-1 has finished reading its stage
+      load(k - 1 + stages, prev);
+    }
+    prev = st;
+    if (++st == stages) {
+      st = 0;
+      phase ^= 1;
+    }
+  }
+  if (lane == 0) bulk_wait_all();
+}
+
 template <bool SP, bool DP>
 cudaError_t launch_t(const CopyArgs& a, int impl, int max_ctas, cudaStream_t s) {
   const uint64_t items_lsu = uint64_t(a.nl) * a.n * ((a.chunk + kLsuPiece - 1) / kLsuPiece);
@@ -233,6 +331,26 @@ cudaError_t launch_t(const CopyArgs& a, int impl, int max_ctas, cudaStream_t s) 
     const uint64_t need = (groups * 32 + kWarpThreads - 1) / kWarpThreads;
     if (grid > need) grid = need;
     copy_warp<SP, DP><<<unsigned(grid), kWarpThreads, 0, s>>>(a);
+  } else if (impl == IMPL_BULKW) {
+    static std::atomic<uint64_t> attr_set_w{0};
+    int dev = 0;
+    cudaError_t e = cudaGetDevice(&dev);
+    if (e != cudaSuccess) return e;
+    const uint64_t bit = 1ull << (dev & 63);
+    if (!(attr_set_w.load() & bit)) {
+      e = cudaFuncSetAttribute(copy_bulkw<SP, DP>, cudaFuncAttributeMaxDynamicSharedMemorySize, kBwSmem);
+      if (e != cudaSuccess) return e;
+      attr_set_w.fetch_or(bit);
+    }
+    // whole chunks up to 16 KiB per stage, larger chunks in pieces; at least 2 stages per warp (the
+    // refill of a stage is issued one item after its store, so one stage would never refill)
+    const uint32_t cap = std::min<uint32_t>(16u << 10, uint32_t(kBwSmem / kBwWarps / 2) & ~15u);
+    const uint32_t piece = a.chunk <= cap ? uint32_t(a.chunk) : cap;
+    const uint64_t items = uint64_t(a.nl) * a.n * ((a.chunk + piece - 1) / piece);
+    uint64_t grid = max_ctas > 0 ? uint64_t(max_ctas) : uint64_t(kSMs);
+    const uint64_t need = (items + kBwWarps - 1) / kBwWarps;  // one item per warp at least
+    if (grid > need) grid = need;
+    copy_bulkw<SP, DP><<<unsigned(grid), kBwWarps * 32, kBwSmem, s>>>(a, piece);
   } else if (impl == IMPL_BULK) {
     static std::atomic<uint64_t> attr_set{0};  // per-device bit: opt-in smem attribute applied
     int dev = 0;
@@ -275,8 +393,11 @@ cudaError_t preload_t() {
   cudaError_t e = cudaFuncGetAttributes(&fa, copy_lsu<SP, DP>);
   if (e == cudaSuccess) e = cudaFuncGetAttributes(&fa, copy_warp<SP, DP>);
   if (e == cudaSuccess) e = cudaFuncGetAttributes(&fa, copy_bulk<SP, DP>);
+  if (e == cudaSuccess) e = cudaFuncGetAttributes(&fa, copy_bulkw<SP, DP>);
   if (e == cudaSuccess)
     e = cudaFuncSetAttribute(copy_bulk<SP, DP>, cudaFuncAttributeMaxDynamicSharedMemorySize, kBulkSmem);
+  if (e == cudaSuccess)
+    e = cudaFuncSetAttribute(copy_bulkw<SP, DP>, cudaFuncAttributeMaxDynamicSharedMemorySize, kBwSmem);
   return e;
 }
 

@@ -24,7 +24,7 @@ struct CopyArgs {
   int32_t l_first = 0;                // absolute layer of t = 0 (paged sides)
 };
 
-enum CopyImpl { IMPL_LSU = 1, IMPL_BULK = 2, IMPL_WARP = 3 };
+enum CopyImpl { IMPL_LSU = 1, IMPL_BULK = 2, IMPL_WARP = 3, IMPL_BULKW = 4 };
 
 // Launch on `s`.  max_ctas <= 0: one full wave of the chosen kernel.  Returns the CUDA error of
 // the launch.  `impl` is IMPL_LSU (registers, 16 B ld.global.nc / st.global) or IMPL_BULK

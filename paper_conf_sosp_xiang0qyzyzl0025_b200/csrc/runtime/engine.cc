@@ -132,6 +132,8 @@ void Ctx::init(int dev, const aeg_config& c) {
   CUDA_TRY(cudaSetDevice(device));
   CUDA_TRY(cudaFree(nullptr));  // create / retain the primary context
   CUDA_TRY(preload_kernels());   // no lazy module load on the data path
+  AEG_REQUIRE(cfg.kernel >= AEG_KERNEL_AUTO && cfg.kernel <= AEG_KERNEL_BULKW, AEG_ERR_INVALID,
+              "unknown kernel selection %d", cfg.kernel);
   AEG_REQUIRE(cfg.staging_slots >= 2, AEG_ERR_INVALID, "need at least 2 staging slots");
   AEG_REQUIRE(cfg.staging_slot_bytes >= 1 * kMiB && cfg.staging_slot_bytes % 256 == 0, AEG_ERR_INVALID,
               "staging slot must be >= 1 MiB and 256-byte aligned");

@@ -228,17 +228,20 @@ static void host_dmas(const SlabPool& hp, char* hbase, const Shape& sh, const st
 // (plain st.global to peer addresses) unless BULK is requested explicitly.
 #define ipc_events(flags) (((flags) & AEG_IPC_EVENTS) || (cfg.flags & AEG_CFG_SHARED_HOST))
 
-// AUTO by chunk size, from tools/launch_probe.cu (profiles/r01/launch_probe2.txt, TB/s body) and
-// tools/threshold_probe.cu (profiles/r01/threshold_probe.txt, ~1 GiB launches, gather / scatter):
-//   2 KiB chunks: WARP 5.1, LSU 1.7, BULK 0.8     8 KiB: LSU 4.8-5.4, WARP 1.5-4.3, BULK 2.7-2.9
-//   16 KiB: LSU 6.0 / 5.9, BULK 5.1 / 5.2         32 KiB: BULK 6.2 / 6.6, LSU 5.8 / 5.8
-//   64-512 KiB: BULK 6.1-6.5, LSU 5.9
+// AUTO by chunk size, from tools/small_chunk_probe.cu (profiles/r02/small_chunk_probe.txt, 1 GiB
+// gather / scatter launches, median TB/s) and tools/threshold_probe.cu (profiles/r01):
+//   2 KiB: WARP 5.96 / 6.01, BULKW 5.63 / 5.62, LSU 1.8, BULK 0.8
+//   4 KiB: BULKW 5.86 / 5.90, WARP 5.57 / 5.62, LSU 3.4-3.5
+//   8 KiB: BULKW 5.98 / 5.91, WARP 5.70 / 5.74, LSU 5.46 / 5.50, BULK 2.99 / 2.93
+//   16 KiB: BULKW 6.04 / 6.00, LSU 6.03 / 5.91, BULK 5.13 / 5.15
+//   32 KiB: BULK 5.98 / 6.14, BULKW 6.03 / 6.00, LSU 5.76 / 5.80;  64-512 KiB: BULK 6.1-6.5, LSU 5.9
 static int impl_of(const aeg_config& cfg, uint64_t chunk) {
   if (cfg.kernel == AEG_KERNEL_LSU) return IMPL_LSU;
   if (cfg.kernel == AEG_KERNEL_BULK) return IMPL_BULK;
   if (cfg.kernel == AEG_KERNEL_WARP) return IMPL_WARP;
-  if (chunk <= (4u << 10)) return IMPL_WARP;
-  return chunk < (32u << 10) ? IMPL_LSU : IMPL_BULK;
+  if (cfg.kernel == AEG_KERNEL_BULKW) return IMPL_BULKW;
+  if (chunk <= (2u << 10)) return IMPL_WARP;
+  return chunk <= (16u << 10) ? IMPL_BULKW : IMPL_BULK;
 }
 
 // ----------------------------------------------------------------------------- swap-out H3

@@ -29,7 +29,7 @@ def _offs(side, sh, handles_o):
     return [OK.addr(side.geom, sh, h, l) for h in handles_o for l in range(sh.L)]
 
 
-@pytest.mark.parametrize("kernel", [aeg.KERNEL_LSU, aeg.KERNEL_BULK])
+@pytest.mark.parametrize("kernel", [aeg.KERNEL_LSU, aeg.KERNEL_BULK, aeg.KERNEL_BULKW])
 def test_host_runs_two_gib_apart_round_trip(kernel):
     require_gpu()
     sh = KVShape(2, 8, 128, 2, 16)          # chunk 64 KiB, block 128 KiB: 8192 blocks per 1 GiB slab

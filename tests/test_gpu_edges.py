@@ -15,11 +15,11 @@ pytestmark = pytest.mark.gpu
 MIB = 1 << 20
 
 
-def make(slot=MIB, dev_slabs=4, host_slabs=4, slab=MIB):
+def make(slot=MIB, dev_slabs=4, host_slabs=4, slab=MIB, kernel=aeg.KERNEL_AUTO):
     cfg = aeg.default_config(device_kv_bytes=dev_slabs * slab, host_kv_bytes=host_slabs * slab, dev_slab_bytes=slab,
                              host_slab_bytes=slab, staging_slot_bytes=slot, staging_slots=2,
                              stage_ring_bytes=4 * MIB, stage_chunk_bytes=MIB, table_arena_bytes=2 * MIB,
-                             host_threads=1)
+                             host_threads=1, kernel=kernel)
     ctx = aeg.Context(0, cfg)
     return ctx, Side(ctx, 0, dev_slabs * slab, slab, 0), Side(ctx, 1, host_slabs * slab, slab, 0)
 
@@ -37,12 +37,13 @@ def test_empty_transfers_are_ready():
         ctx.shutdown()
 
 
+@pytest.mark.parametrize("kernel", [aeg.KERNEL_AUTO, aeg.KERNEL_BULKW, aeg.KERNEL_BULK, aeg.KERNEL_LSU])
 @pytest.mark.parametrize("shape", [(1, 1, 8, 2, 1), (3, 1, 8, 2, 1), (1, 2, 64, 2, 16)])
-def test_small_shapes_round_trip(shape):
+def test_small_shapes_round_trip(shape, kernel):
     """One-layer shapes and 1-token blocks (chunk = 32 B): ragged, launch-bound, still bit-exact."""
     require_gpu()
     sh = KVShape(*shape)
-    ctx, dev, host = make()
+    ctx, dev, host = make(kernel=kernel)
     try:
         dev.poison(gi.TAG_NEVER)
         host.poison(gi.TAG_NEVER)

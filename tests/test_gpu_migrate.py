@@ -29,7 +29,7 @@ def make(layout, slab=MIB, nslabs=8, kernel=aeg.KERNEL_LSU):
     return ctx, Side(ctx, aeg.POOL_DEVICE, cfg.device_kv_bytes, slab, layout)
 
 
-@pytest.mark.parametrize("kernel", [aeg.KERNEL_LSU, aeg.KERNEL_BULK])
+@pytest.mark.parametrize("kernel", [aeg.KERNEL_LSU, aeg.KERNEL_BULK, aeg.KERNEL_BULKW])
 def test_local_migrate(kernel):
     require_gpu()
     ctx, dev = make(aeg.BLOCK_MAJOR, kernel=kernel)

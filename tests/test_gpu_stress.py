@@ -35,7 +35,7 @@ def test_random_overlapping_transfers(seed):
                              host_slab_bytes=256 * KIB, dev_slab_layout=seed % 2, host_slab_layout=(seed // 2) % 2,
                              staging_slot_bytes=1 << 20, staging_slots=2, stage_ring_bytes=4 << 20,
                              stage_chunk_bytes=1 << 20, device_weight_bytes=2 << 20, table_arena_bytes=2 << 20,
-                             host_threads=1, kernel=aeg.KERNEL_BULK if seed % 3 else aeg.KERNEL_LSU)
+                             host_threads=1, kernel=[aeg.KERNEL_LSU, aeg.KERNEL_BULK, aeg.KERNEL_BULKW][seed % 3])
     _stress(seed, cfg, SH, 12)
 
 

@@ -64,7 +64,7 @@ LAYOUTS = [(aeg.LAYER_MAJOR, aeg.LAYER_MAJOR), (aeg.BLOCK_MAJOR, aeg.LAYER_MAJOR
            (aeg.LAYER_MAJOR, aeg.BLOCK_MAJOR), (aeg.BLOCK_MAJOR, aeg.BLOCK_MAJOR)]
 
 
-@pytest.mark.parametrize("kernel", [aeg.KERNEL_LSU, aeg.KERNEL_BULK, aeg.KERNEL_WARP])
+@pytest.mark.parametrize("kernel", [aeg.KERNEL_LSU, aeg.KERNEL_BULK, aeg.KERNEL_WARP, aeg.KERNEL_BULKW])
 @pytest.mark.parametrize("layouts", LAYOUTS)
 @pytest.mark.parametrize("slot", [1 << 20, 8 << 20])
 def test_c1_round_trip_full_images(layouts, kernel, slot):

@@ -1,0 +1,114 @@
+// Small-chunk gather/scatter probe: event-timed back-to-back launches of the product
+// copy kernels (csrc/kernels/copy.cu, included verbatim; BULKW geometry set by -D) on scattered
+// block tables, for 2-32 KiB chunks, gather (paged -> contiguous) and scatter (contiguous -> paged).
+// GB/s = algorithmic bytes (2 x payload) / median event time.
+// Build: nvcc -gencode arch=compute_100a,code=sm_100a -O3 -DAEG_BW_WARPS=4 -DAEG_BW_SMEM_KIB=192 \
+//          -o build/small_chunk_probe tools/small_chunk_probe.cu
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <cstdlib>
+#include <cstdio>
+#include <vector>
+
+#include "../paper_conf_sosp_xiang0qyzyzl0025_b200/csrc/kernels/copy.cu"
+
+int main() {
+  const uint64_t payload = 1ull << 30;  // 1 GiB per launch each way
+  for (uint64_t chunk : {2048ull, 4096ull, 8192ull, 16384ull, 32768ull}) {
+    const int n = int(payload / chunk);
+    char *pool, *slot;
+    cudaMalloc(&pool, 2 * payload);  // blocks scattered over twice the payload
+    cudaMalloc(&slot, payload);
+    std::vector<uint64_t> off(n);
+    for (int i = 0; i < n; ++i) off[i] = uint64_t((uint64_t(i) * 7919) % (2 * n)) * chunk;
+    std::sort(off.begin(), off.end());
+    off.erase(std::unique(off.begin(), off.end()), off.end());
+    while (int(off.size()) < n) off.push_back(off.back() + chunk);
+    for (int i = n - 1; i > 0; --i) std::swap(off[i], off[(uint64_t(i) * 2654435761u) % (i + 1)]);
+    uint64_t* doff;
+    cudaMalloc(&doff, n * 8);
+    cudaMemcpy(doff, off.data(), n * 8, cudaMemcpyHostToDevice);
+    cudaStream_t s;
+    cudaStreamCreateWithFlags(&s, cudaStreamNonBlocking);
+    cudaEvent_t a, b;
+    cudaEventCreate(&a);
+    cudaEventCreate(&b);
+    for (int dir = 0; dir < 2; ++dir) {
+      aeg::CopyArgs ca;
+      if (dir == 0) {
+        ca.src = pool;
+        ca.src_off = doff;
+        ca.dst = slot;
+      } else {
+        ca.src = slot;
+        ca.dst = pool;
+        ca.dst_off = doff;
+      }
+      ca.src_lstride = ca.dst_lstride = chunk;
+      ca.chunk = chunk;
+      ca.nl = 1;
+      ca.n = n;
+      if (getenv("SWEEP")) {  // BULKW with explicit piece sizes (chunk / 2^k, >= 1 KiB, >= 2 stages)
+        using namespace aeg;
+        cudaFuncSetAttribute(copy_bulkw<true, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, kBwSmem);
+        cudaFuncSetAttribute(copy_bulkw<false, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, kBwSmem);
+        for (uint64_t piece = chunk; piece >= 1024; piece /= 2) {
+          if (piece * 2 > uint64_t(kBwSmem / kBwWarps)) continue;
+          const uint64_t items = uint64_t(n) * ((chunk + piece - 1) / piece);
+          const int smp = 2 * 1024 * 1024 / 1;  // unused
+          (void)smp;
+          int occ = 0;
+          cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, copy_bulkw<true, false>, kBwWarps * 32, kBwSmem);
+          uint64_t grid = uint64_t(148) * std::max(1, occ);
+          if (grid > (items + kBwWarps - 1) / kBwWarps) grid = (items + kBwWarps - 1) / kBwWarps;
+          std::vector<float> ts;
+          for (int r = 0; r < 12; ++r) {
+            cudaEventRecord(a, s);
+            if (dir == 0)
+              copy_bulkw<true, false><<<unsigned(grid), kBwWarps * 32, kBwSmem, s>>>(ca, uint32_t(piece));
+            else
+              copy_bulkw<false, true><<<unsigned(grid), kBwWarps * 32, kBwSmem, s>>>(ca, uint32_t(piece));
+            cudaEventRecord(b, s);
+            cudaEventSynchronize(b);
+            float ms;
+            cudaEventElapsedTime(&ms, a, b);
+            if (r >= 2) ts.push_back(ms);
+          }
+          std::sort(ts.begin(), ts.end());
+          const double med = ts[ts.size() / 2];
+          printf("chunk=%6llu %s BULKW warps=%d smem=%dK ctas/SM=%d piece=%6llu median %8.1f us  %7.0f GB/s\n",
+                 (unsigned long long)chunk, dir ? "scatter" : "gather ", kBwWarps, kBwSmem >> 10, occ,
+                 (unsigned long long)piece, med * 1e3, 2.0 * payload / (med * 1e6));
+        }
+        continue;
+      }
+      for (int impl : {aeg::IMPL_LSU, aeg::IMPL_WARP, aeg::IMPL_BULK, aeg::IMPL_BULKW}) {
+        std::vector<float> ts;
+        for (int r = 0; r < 12; ++r) {
+          cudaEventRecord(a, s);
+          cudaError_t e = aeg::launch_copy(ca, impl, 0, s);
+          cudaEventRecord(b, s);
+          cudaEventSynchronize(b);
+          if (e != cudaSuccess || cudaGetLastError() != cudaSuccess) {
+            printf("error %s\n", cudaGetErrorString(e));
+            return 1;
+          }
+          float ms;
+          cudaEventElapsedTime(&ms, a, b);
+          if (r >= 2) ts.push_back(ms);
+        }
+        std::sort(ts.begin(), ts.end());
+        const double med = ts[ts.size() / 2];
+        printf("chunk=%6llu %s %-5s median %8.1f us  %7.0f GB/s (best %7.0f)\n", (unsigned long long)chunk,
+               dir ? "scatter" : "gather ",
+               impl == aeg::IMPL_LSU ? "LSU" : impl == aeg::IMPL_WARP ? "WARP" : impl == aeg::IMPL_BULK ? "BULK" : "BULKW",
+               med * 1e3, 2.0 * payload / (med * 1e6), 2.0 * payload / (ts[0] * 1e6));
+      }
+    }
+    cudaFree(pool);
+    cudaFree(slot);
+    cudaFree(doff);
+  }
+  return 0;
+}
