@@ -98,7 +98,10 @@ typedef struct {
 
 /* Sizes are bytes.  Zero fields take the defaults of aeg_config_default(). */
 typedef struct {
-  uint64_t device_kv_bytes;     /* unified GPU KV cache region (slabs)                        */
+  uint64_t device_kv_bytes;     /* unified GPU KV cache region (slabs).  0 = the paper's sizing
+                                   (reading 22): the one device allocation
+                                   takes 90% of free VRAM, the KV region gets what the other
+                                   regions leave, in whole slabs (aeg_pool_region reports it)   */
   uint64_t device_weight_bytes; /* self-managed weights region (bump allocated)               */
   uint64_t host_kv_bytes;       /* unified CPU KV cache, pinned once at init  */
   uint64_t dev_slab_bytes;      /* slab size of the device pool          */
@@ -185,8 +188,10 @@ int aeg_kv_alloc(aeg_ctx ctx, int32_t pool, const aeg_kv_shape* shape, int32_t n
  * nothing is freed. */
 int aeg_kv_free(aeg_ctx ctx, int32_t pool, const aeg_block* blocks, int32_t n);
 
-/* Release move-list blocks whose transfers completed.  blocking != 0 first waits for every
- * in-flight transfer.  Returns AEG_OK. */
+/* Step ⑧ on demand (§5.3: "a daemon thread periodically queries
+ * (cudaEventQuery) events in the move lists to reclaim the blocks once the transfers complete"):
+ * release move-list blocks whose transfers completed, reap released transfers.  blocking != 0
+ * first waits for every in-flight transfer.  Returns AEG_OK. */
 int aeg_reclaim(aeg_ctx ctx, int blocking);
 
 /* Pool statistics.  Fig. 16's fragmentation, "the ratio of unused memory to peak allocated memory"
@@ -196,8 +201,10 @@ int aeg_stats(aeg_ctx ctx, int32_t pool, aeg_pool_stats* out);
 /* Decode a handle.  Any output pointer may be NULL. */
 int aeg_block_info(aeg_ctx ctx, aeg_block b, int32_t* pool, uint32_t* slab, uint32_t* index);
 
-/* Address of layer `layer` of block b: device pointer (device pool) or host pointer (host pool,
- * pinned and device-mapped).  The block must be owned and of `shape`. */
+/* Address of layer `layer` of block b inside its slab (§5.2: a slab "serving as
+ * a pool of KV cache blocks for that specific shape"; the in-slab layout is reading 5): device
+ * pointer (device pool) or host pointer (host pool, pinned and device-mapped).  The block must be
+ * owned and of `shape`; INVALID otherwise.  *p is written only on AEG_OK. */
 int aeg_block_ptr(aeg_ctx ctx, int32_t pool, const aeg_kv_shape* shape, aeg_block b,
                   int32_t layer, void** p);
 
@@ -235,7 +242,9 @@ int aeg_kv_swap_out(aeg_ctx ctx, const aeg_kv_shape* shape, const aeg_block* dev
 int aeg_kv_swap_in(aeg_ctx ctx, const aeg_kv_shape* shape, const aeg_block* host,
                    const aeg_block* dev, int32_t n, uint32_t flags, aeg_xfer* out);
 
-/* Prefill->decode hand-off: dst_pool_of(peer)[addr_dst(dst[i], l)] = dev[addr_src(src[i], l)] for
+/* Prefill->decode hand-off (north star; Fig. 10, the KV of a request moving from
+ * a prefill instance to a decoding instance, here directly GPU-to-GPU instead of through the CPU
+ * cache): dst_pool_of(peer)[addr_dst(dst[i], l)] = dev[addr_src(src[i], l)] for
  * every layer, by a fused kernel on this GPU that reads local blocks and stores 16-byte vectors
  * straight into the peer's pool over NVLink/NVSwitch (no staging).  `peer` is an index given to
  * aeg_import_peer, or -1 for this context's own device pool (local relocation).  dst handles are
@@ -275,7 +284,9 @@ int aeg_layer_ready(aeg_ctx ctx, aeg_xfer x, int32_t layer, int32_t mode, void* 
 /* Number of readiness layers of x. */
 int aeg_xfer_layers(aeg_ctx ctx, aeg_xfer x, int32_t* layers);
 
-/* The caller will not query x again; its events are recycled once it completes. */
+/* The caller will not query x again; its CUDA events (Table 2) are recycled
+ * once it completes (and, for a transfer imported by another context of this process, once that
+ * import is reaped).  STATE for an unknown transfer. */
 int aeg_xfer_release(aeg_ctx ctx, aeg_xfer x);
 
 /* ---- weights (H7, N1) ----------------------------------------------------------------------- */
@@ -321,12 +332,16 @@ int aeg_host_unregister(aeg_ctx ctx, void* ptr);
 /* ---- multi-process (H5) ------------------------------------------------------------------- */
 
 /* Serialise this context's device-pool IPC handle, geometry and interprocess event ring into
- * buf (capacity *len in, bytes used out).  buf == NULL: *len receives the required size. */
+ * buf (capacity *len in, bytes used out).  buf == NULL: *len receives the required size.
+ * PAPER.md:1528-1532 §5.3 ("Events are also passed between instances via interprocess
+ * communication (IPC) for synchronizing different instances"; cudaIpcGetEventHandle, Table 2). */
 int aeg_export_ipc(aeg_ctx ctx, void* buf, uint64_t* len);
 
 /* Map a peer's device pool (cudaIpcOpenMemHandle, or a direct pointer when the peer lives in
- * this process) and its event ring, and enable peer access.  `peer` is the caller's index for
- * it (0..63). */
+ * this process) and its event ring (cudaIpcOpenEventHandle, Table 2), and
+ * enable peer access when the peer is another GPU.  `peer` is the caller's index for it (0..63);
+ * importing an index again replaces that peer's mappings.  INVALID for a malformed blob or index,
+ * STATE in a host-only context, CUDA when the mapping or peer access fails. */
 int aeg_import_peer(aeg_ctx ctx, int32_t peer, const void* buf, uint64_t len);
 
 /* Serialise transfer x's per-layer interprocess events (after it was enqueued) so the peer can

@@ -116,11 +116,31 @@ void unmap_shared_host(char* b, uint64_t bytes) {
 }
 
 // ------------------------------------------------------------------------------------ init
+constexpr double kVramReserveFrac = 0.10;  // left free for the caller's tensors
+
 void Ctx::init(int dev, const aeg_config& c) {
   cfg = c;
   host_only = (cfg.flags & AEG_CFG_HOST_ONLY) != 0;
   timing = (cfg.flags & AEG_CFG_TIMING) != 0;
   AEG_REQUIRE(cfg.dev_slab_bytes > 0 && cfg.host_slab_bytes > 0, AEG_ERR_INVALID, "slab sizes must be > 0");
+  if (!host_only && cfg.device_kv_bytes == 0) {
+    // Reading 22: the self-managed buffer takes "all the necessary VRAM ... in
+    // one allocation, leaving around 10% free memory for tensor libraries".  device_kv_bytes = 0
+    // sizes the KV region so that the whole allocation (KV + weights + staging rings + tables) is
+    // 90% of the device's free memory, rounded down to whole slabs.
+    CUDA_TRY(cudaSetDevice(dev));
+    CUDA_TRY(cudaFree(nullptr));
+    size_t fr = 0, tot = 0;
+    CUDA_TRY(cudaMemGetInfo(&fr, &tot));
+    const uint64_t others = align_up(cfg.device_weight_bytes, kAlign) +
+                            2 * align_up(cfg.staging_slot_bytes * uint64_t(cfg.staging_slots), kAlign) +
+                            align_up(cfg.table_arena_bytes, kAlign);
+    const uint64_t budget = uint64_t(double(fr) * (1.0 - kVramReserveFrac));
+    AEG_REQUIRE(budget > others + cfg.dev_slab_bytes, AEG_ERR_OOM,
+                "90%% of free VRAM (%llu bytes) does not hold the other regions plus one slab",
+                (unsigned long long)budget);
+    cfg.device_kv_bytes = (budget - others) / cfg.dev_slab_bytes * cfg.dev_slab_bytes;
+  }
   pool[AEG_POOL_DEVICE].init(AEG_POOL_DEVICE, cfg.device_kv_bytes, cfg.dev_slab_bytes, cfg.dev_slab_layout);
   pool[AEG_POOL_HOST].init(AEG_POOL_HOST, cfg.host_kv_bytes, cfg.host_slab_bytes, cfg.host_slab_layout);
   for (auto& p : pool) p.is_done = [this](uint64_t x) { return is_done(x); };

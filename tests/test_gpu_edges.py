@@ -143,3 +143,27 @@ def test_swap_sources_must_be_owned_and_distinct():
         assert e.value.code in (aeg.ERR_STATE, aeg.ERR_INVALID)
     finally:
         ctx.shutdown()
+
+
+def test_default_device_kv_takes_90pct_of_free_vram():
+    """Reading 22: device_kv_bytes = 0 sizes the one device allocation to ~90% of
+    free VRAM ("leaving around 10% free memory for tensor libraries"), the KV region in whole slabs."""
+    require_gpu()
+    import torch
+    free0, _ = torch.cuda.mem_get_info()
+    cfg = aeg.default_config(device_kv_bytes=0, host_kv_bytes=4 * MIB, dev_slab_bytes=64 * MIB,
+                             host_slab_bytes=MIB, staging_slot_bytes=MIB, staging_slots=2,
+                             stage_ring_bytes=4 * MIB, stage_chunk_bytes=MIB, device_weight_bytes=256 * MIB,
+                             table_arena_bytes=2 * MIB, host_threads=1)
+    ctx = aeg.Context(0, cfg)
+    try:
+        _, kv = ctx.pool_region(aeg.POOL_DEVICE)
+        others = 256 * MIB + 2 * 2 * MIB + 2 * MIB
+        assert kv % (64 * MIB) == 0 and kv > 0
+        assert 0.9 * free0 - others - 64 * MIB - 256 * MIB <= kv <= 0.9 * free0 - others
+        free1, _ = torch.cuda.mem_get_info()
+        assert free1 >= 0.09 * free0            # ~10% left to the caller
+        b = ctx.kv_alloc(aeg.POOL_DEVICE, (2, 4, 64, 2, 16), 8)
+        ctx.kv_free(aeg.POOL_DEVICE, b)
+    finally:
+        ctx.shutdown()
