@@ -117,6 +117,9 @@ class Dist:
         if world > 1:
             import torch.distributed as td
             os.environ.setdefault("MASTER_ADDR", "127.0.0.1")
+            # NCCL's init lines (comm ... nRanks N) in the log let the driver count the ranks
+            os.environ.setdefault("NCCL_DEBUG", "INFO")
+            os.environ.setdefault("NCCL_DEBUG_SUBSYS", "INIT")
             if self.backend == "nccl":
                 td.init_process_group("nccl", device_id=torch.device("cuda", self.device))
             else:
@@ -1031,6 +1034,75 @@ def migrate_leg(aeg, torch, kernel, n_req=16, src_layout=None, dst_layout=None):
             "per_chunk_memcpy_calls": int(len(offs))}
 
 
+def migrate_leg_two_device(aeg, torch, kernel, n_req=16):
+    """configs[2] between two GPUs of ONE process (rank 0 of an N >= 2 run, every GPU visible): the
+    prefill context on cuda:0 migrates n_req Llama-2-13B requests into the pool of a decode context
+    on cuda:1 mapped directly (aeg_import_peer's same-process cross-device branch:
+    cudaDeviceEnablePeerAccess, 16-byte stores into the peer aperture over NVLink).  Reports GB/s
+    by CTA budget and the smallest budget reaching 0.70 x 900 GB/s; bit-exact at the destination."""
+    import aeg_inputs as gi
+    from aeg_inputs import dev as D
+    if torch.cuda.device_count() < 2:
+        return {"skipped": "needs two visible GPUs"}
+    sht = gi.KV_SHAPES["llama-2-13b"]
+    sh = aeg.KVShape.of(sht)
+    lens = gi.request_lengths(3, n_req, 512, 4096)
+    n = sum(-(-t // 16) for t in lens)
+    slab = GIB + 256 * MIB
+    nslab = -(-n // (slab // sh.block_bytes())) + 1
+    mk = lambda dev, lay: aeg.Context(dev, aeg.default_config(  # noqa: E731
+        device_kv_bytes=nslab * slab, host_kv_bytes=GIB, dev_slab_bytes=slab, dev_slab_layout=lay, kernel=kernel,
+        flags=aeg.CFG_TIMING))
+    a = mk(0, aeg.LAYER_MAJOR)
+    b = mk(1, aeg.BLOCK_MAJOR)
+    try:
+        sc, dc = a.kv_alloc(0, sht, n), b.kv_alloc(0, sht, n)
+        abase, _ = a.pool_region(0)
+        bbase, _ = b.pool_region(0)
+        seed = gi.kv_seed(3)
+        keys = [gi.kv_key(1, 7, i, l) for i in range(n) for l in range(sh.num_layers)]
+        torch.cuda.set_device(0)
+        D.fill_chunks(abase, chunk_offsets(a, 0, sht, sc), keys, sh.chunk_bytes(), seed)
+        D.sync()
+        a.import_peer(1, b.export_ipc())
+        s = torch.cuda.Stream(device=0)
+
+        def timed(reps):
+            out = []
+            for it in range(reps + 1):
+                e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                e0.record(s)
+                a.stream_fence(s.cuda_stream)
+                x = a.kv_migrate(sht, sc, 1, dc)
+                a.layer_ready(x, -1, aeg.READY_WAIT_STREAM, s.cuda_stream)
+                e1.record(s)
+                e1.synchronize()
+                a.xfer_release(x)
+                if it:
+                    out.append(e0.elapsed_time(e1))
+            return out
+        payload = n * sh.block_bytes()
+        sweep = {}
+        for ctas in (8, 16, 32, 48, 64, 96, 148):
+            a.set_migrate_ctas(ctas)
+            sweep[ctas] = round(payload / (min(timed(2)) * 1e6), 1)
+        a.set_migrate_ctas(0)
+        ms = statistics.median(timed(4))
+        torch.cuda.set_device(1)
+        bad, _ = D.verify_chunks(bbase, chunk_offsets(b, 0, sht, dc), keys, sh.chunk_bytes(), seed)
+        torch.cuda.set_device(0)
+        ok = [c for c, v in sorted(sweep.items()) if v >= 0.70 * NVLINK_NOMINAL]
+        return {"workload": f"configs[2] Llama-2-13B hand-off, {n_req} requests ({n} blocks), cuda:0 -> cuda:1 in "
+                            "one process (direct peer mapping, NVLink)",
+                "payload_bytes": payload, "ms": round(ms, 3), "GBps": round(payload / (ms * 1e6), 1),
+                "frac_of_nvlink_nominal": round(payload / (ms * 1e6) / NVLINK_NOMINAL, 3),
+                "GBps_by_ctas": sweep, "ctas_for_70pct_nvlink": ok[0] if ok else None, "bit_exact": bad == 0}
+    finally:
+        torch.cuda.set_device(0)
+        a.shutdown()
+        b.shutdown()
+
+
 def _nccl_sendrecv(torch, dist, pairs, nbytes, reps=4):
     """NCCL point-to-point of one hand-off's payload as ONE contiguous buffer per pair (no block
     tables, no gather/scatter: an upper bound for an NCCL-based hand-off).  Max-over-ranks device
@@ -1128,6 +1200,8 @@ def migrate_leg_dist(aeg, torch, dist, kernel, n_req=16):
         ctx.set_migrate_ctas(ctas)
         sweep[ctas] = round(len(pairs) * n * sh.block_bytes() / (min(hand_off(pairs) for _ in range(2)) * 1e6), 1)
     ctx.set_migrate_ctas(0)
+    per_pair_target = 0.70 * NVLINK_NOMINAL
+    ok_ctas = [c for c, v in sorted(sweep.items()) if v / len(pairs) >= per_pair_target]
     bad = 0
     if not prefill:
         sender = [s_ for s_, d in pairs if d == rank][0]
@@ -1186,6 +1260,7 @@ def migrate_leg_dist(aeg, torch, dist, kernel, n_req=16):
             "frac_of_measured_peer_copy_per_pair": round(payload / len(pairs) / (ms * 1e6) / NVLINK_PEER_COPY, 3),
             "kernel_GBps_payload_max_rank": round(k_gbps, 1), "kernel_launches_per_xfer": int(kl // 5) if kl else 0,
             "GBps_aggregate_by_ctas": sweep,
+            "ctas_for_70pct_nvlink_per_pair": ok_ctas[0] if ok_ctas else None,
             "bit_exact": bad == 0, "all_to_all": a2a}
 
 
@@ -1294,6 +1369,20 @@ def host_route_leg(aeg, torch, kernel, n_req=4, reps=4):
             raise RuntimeError("decode process handshake")
         ts = torch.zeros(2, dtype=torch.int64, device="cuda")
         s, s2 = new_stream(torch), new_stream(torch)
+        alone = []   # P->C with no concurrent C->D: the shared region's one-direction rate
+        for _ in range(3):
+            hc = a.kv_alloc(1, sht, n)
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record(s)
+            a.stream_fence(s.cuda_stream)
+            xo = a.kv_swap_out(sht, src, hc)
+            a.layer_ready(xo, -1, aeg.READY_WAIT_STREAM, s.cuda_stream)
+            e1.record(s)
+            e1.synchronize()
+            alone.append(e0.elapsed_time(e1))
+            a.xfer_release(xo)
+            a.kv_free(1, hc)
+            a.reclaim(True)
         gate = D.Gate()
         for _ in range(reps + 1):
             hc = a.kv_alloc(1, sht, n)
@@ -1331,7 +1420,13 @@ def host_route_leg(aeg, torch, kernel, n_req=4, reps=4):
     return {"workload": f"configs[2] Llama-2-13B hand-off of {n_req} requests ({n} blocks, {b / GIB:.2f} GiB) through "
                         "the node-shared pinned CPU cache, P and D in two processes on one GPU",
             "p_to_c_ms": round(out_ns / 1e6, 2), "p_to_c_GBps": round(b / out_ns, 1),
+            "p_to_c_alone_GBps": round(b / (min(alone[1:]) * 1e6), 1),
+            "p_to_c_alone_frac_of_pcie_nominal": round(b / (min(alone[1:]) * 1e6) / PCIE_NOMINAL, 3),
             "p_to_d_ms": round(e2e_ns / 1e6, 2), "p_to_d_GBps": round(b / e2e_ns, 1),
+            "both_directions_GBps_over_p_to_d": round(2 * b / e2e_ns, 1),
+            "note": "P->C and C->D overlap layer by layer, so p_to_c_GBps is one direction of a duplex "
+                    "transfer (this box's duplex memcpy ceiling is in pcie_memcpy_GBps.bidir_total); "
+                    "p_to_c_alone_GBps is the same swap-out into the shared region with D idle",
             "bit_exact": all(r[2] == 0 for r in res), "reps": len(res)}
 
 
@@ -1863,6 +1958,10 @@ def run_ours(args):
             mig = None
         elif world > 1:
             mig = leg("migrate", lambda: migrate_leg_dist(aeg, torch, dist, kernel, args.migrate_requests))
+            if rank == 0 and dist.local == 0:   # the cross-device branch of aeg_import_peer, one process
+                mig["two_device_same_process"] = leg("migrate_two_device",
+                                                     lambda: migrate_leg_two_device(aeg, torch, kernel))
+            dist.barrier()
         else:
             mig = leg("migrate", lambda: migrate_leg(aeg, torch, kernel, args.migrate_requests))
         sw = None

@@ -325,3 +325,44 @@ def test_two_process_host_route_p_c_d(nblocks):
         if p.is_alive():
             p.kill()
     assert p.exitcode == 0
+
+
+def test_two_device_same_process_migrate():
+    """H5 across two GPUs of one process (aeg_import_peer's same-process cross-device branch: peer
+    access enabled, the migrate kernel on cuda:0 stores into cuda:1's pool over NVLink): the
+    destination image equals oracle.kv.migrate (O7).  Needs two visible GPUs."""
+    require_gpu()
+    import torch
+    if torch.cuda.device_count() < 2:
+        pytest.skip("needs two visible GPUs")
+    cfg = lambda lay, slab: aeg.default_config(  # noqa: E731
+        device_kv_bytes=6 * slab, host_kv_bytes=MIB, dev_slab_bytes=slab, host_slab_bytes=MIB,
+        dev_slab_layout=lay, staging_slot_bytes=MIB, staging_slots=2, stage_ring_bytes=4 * MIB,
+        stage_chunk_bytes=MIB, table_arena_bytes=2 * MIB, host_threads=1, kernel=aeg.KERNEL_LSU)
+    a = aeg.Context(0, cfg(aeg.LAYER_MAJOR, MIB))
+    b = aeg.Context(1, cfg(aeg.BLOCK_MAJOR, MIB + 64 * 1024))
+    try:
+        A = Side(a, aeg.POOL_DEVICE, 6 * MIB, MIB, aeg.LAYER_MAJOR)
+        torch.cuda.set_device(1)
+        B = Side(b, aeg.POOL_DEVICE, 6 * (MIB + 64 * 1024), MIB + 64 * 1024, aeg.BLOCK_MAJOR)
+        B.poison(gi.TAG_NEVER)
+        bimg = B.poison_img(gi.TAG_NEVER)
+        dc, do = B.alloc(SH, 50)
+        poison_blocks(B, bimg, SH, do)
+        torch.cuda.set_device(0)
+        A.poison(gi.TAG_NEVER)
+        aimg = A.poison_img(gi.TAG_NEVER)
+        sc, so = A.alloc(SH, 50)
+        fill_blocks(A, aimg, SH, so, [(4, j) for j in range(50)])
+        a.import_peer(1, b.export_ipc())
+        x = a.kv_migrate(SH.as_tuple(), sc, 1, dc)
+        a.layer_ready(x, -1, aeg.READY_BLOCK)
+        exp = OK.migrate(aimg, A.geom, bimg, B.geom, SH, so, do)
+        torch.cuda.set_device(1)
+        assert first_diff(B.read(), exp) is None
+        torch.cuda.set_device(0)
+        assert first_diff(A.read(), aimg) is None
+    finally:
+        torch.cuda.set_device(0)
+        a.shutdown()
+        b.shutdown()
