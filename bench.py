@@ -59,7 +59,7 @@ def parse():
     p.add_argument("--warmup", type=int, default=3)
     p.add_argument("--impl", default="ours", choices=["ours", "reference"])
     p.add_argument("--requests", type=int, default=64)
-    p.add_argument("--kernel", default="auto", choices=["auto", "lsu", "bulk"])
+    p.add_argument("--kernel", default="auto", choices=["auto", "lsu", "bulk", "bulkw", "warp"])
     p.add_argument("--no-switch", action="store_true")
     p.add_argument("--no-migrate", action="store_true")
     p.add_argument("--no-c5", action="store_true", help="skip the configs[4] Qwen-72B TP=4 scale-up leg")
@@ -1846,7 +1846,8 @@ def run_ours(args):
         build.build()
     dist = Dist(world, rank, local)
     dist.barrier()
-    kernel = {"auto": aeg.KERNEL_AUTO, "lsu": aeg.KERNEL_LSU, "bulk": aeg.KERNEL_BULK}[args.kernel]
+    kernel = {"auto": aeg.KERNEL_AUTO, "lsu": aeg.KERNEL_LSU, "bulk": aeg.KERNEL_BULK, "bulkw": aeg.KERNEL_BULKW,
+              "warp": aeg.KERNEL_WARP}[args.kernel]
     n_req = args.requests
     if world > 1:   # keep the pinned host pools inside host RAM when several ranks share a node
         import psutil

@@ -574,13 +574,16 @@ uint64_t Ctx::migrate(const Shape& sh, const aeg_block* src, int32_t peer, const
   const uint64_t layer = uint64_t(n) * sh.chunk();
   int32_t lps = 1;
   if (n > 0 && layer < pack) lps = int32_t(std::min<uint64_t>(sh.L, std::max<uint64_t>(1, pack / layer)));
-  // Paged -> paged under AUTO: LSU (WARP for tiny chunks), local or remote.  Remote: plain st.global
-  // to the peer aperture, never bulk copies.  Local: with both sides paged the BULK ring loses to
-  // LSU once the pools span tens of GB (profiles/r01/migrate_probe.txt: 16 Llama-2-13B requests,
-  // 30 GB per side: LSU 5.44-5.84 TB/s vs BULK 5.02-5.19 over all four layout pairs; 4 requests:
-  // BULK 2-3 % ahead).
-  const int impl = cfg.kernel == AEG_KERNEL_AUTO ? (sh.chunk() <= (4u << 10) ? IMPL_WARP : IMPL_LSU)
-                                                 : impl_of(cfg, sh.chunk());
+  // Paged -> paged under AUTO (WARP for tiny chunks).  Remote: LSU, plain st.global to the peer
+  // aperture (bulk copies into another GPU's memory are not relied on).  Local: BULKW — with both
+  // sides paged over tens of GB the single-issuer BULK ring loses to LSU, the 4-issuer BULKW beats
+  // both (profiles/r02/migrate_leg_probe_r02.txt, 16 Llama-2-13B requests, 30 GB per side, the four
+  // layout pairs: BULKW 5.54-5.96 TB/s, LSU 5.36-5.82, BULK 5.02-5.22; 4 requests: BULKW 5.44-5.61,
+  // BULK 5.38-5.66, LSU 5.34-5.53).
+  const int impl = cfg.kernel != AEG_KERNEL_AUTO ? impl_of(cfg, sh.chunk())
+                   : sh.chunk() <= (4u << 10)    ? IMPL_WARP
+                   : remote                      ? IMPL_LSU
+                                                 : IMPL_BULKW;
   for (int32_t la = 0; la < sh.L; la += lps) {
     const int32_t lb = std::min(sh.L, la + lps);
     if (n > 0) {

@@ -15,7 +15,10 @@
 
 int main() {
   const uint64_t payload = 1ull << 30;  // 1 GiB per launch each way
-  for (uint64_t chunk : {2048ull, 4096ull, 8192ull, 16384ull, 32768ull}) {
+  const bool mig = getenv("MIGRATE") != nullptr;  // paged -> paged (H5 local) at large chunks
+  std::vector<uint64_t> chunks = {2048ull, 4096ull, 8192ull, 16384ull, 32768ull};
+  if (mig) chunks = {32768ull, 262144ull, 327680ull};
+  for (uint64_t chunk : chunks) {
     const int n = int(payload / chunk);
     char *pool, *slot;
     cudaMalloc(&pool, 2 * payload);  // blocks scattered over twice the payload
@@ -34,9 +37,23 @@ int main() {
     cudaEvent_t a, b;
     cudaEventCreate(&a);
     cudaEventCreate(&b);
-    for (int dir = 0; dir < 2; ++dir) {
+    uint64_t* doff2 = nullptr;
+    char* pool2 = nullptr;
+    if (mig) {  // a second scattered table into a second pool
+      std::vector<uint64_t> off2(off);
+      for (int i = n - 1; i > 0; --i) std::swap(off2[i], off2[(uint64_t(i) * 40503u + 7) % (i + 1)]);
+      cudaMalloc(&doff2, n * 8);
+      cudaMemcpy(doff2, off2.data(), n * 8, cudaMemcpyHostToDevice);
+      cudaMalloc(&pool2, 2 * payload);
+    }
+    for (int dir = 0; dir < (mig ? 1 : 2); ++dir) {
       aeg::CopyArgs ca;
-      if (dir == 0) {
+      if (mig) {
+        ca.src = pool;
+        ca.src_off = doff;
+        ca.dst = pool2;
+        ca.dst_off = doff2;
+      } else if (dir == 0) {
         ca.src = pool;
         ca.src_off = doff;
         ca.dst = slot;
@@ -78,7 +95,7 @@ int main() {
           std::sort(ts.begin(), ts.end());
           const double med = ts[ts.size() / 2];
           printf("chunk=%6llu %s BULKW warps=%d smem=%dK ctas/SM=%d piece=%6llu median %8.1f us  %7.0f GB/s\n",
-                 (unsigned long long)chunk, dir ? "scatter" : "gather ", kBwWarps, kBwSmem >> 10, occ,
+                 (unsigned long long)chunk, mig ? "migrate" : dir ? "scatter" : "gather ", kBwWarps, kBwSmem >> 10, occ,
                  (unsigned long long)piece, med * 1e3, 2.0 * payload / (med * 1e6));
         }
         continue;
@@ -109,6 +126,10 @@ int main() {
     cudaFree(pool);
     cudaFree(slot);
     cudaFree(doff);
+    if (mig) {
+      cudaFree(pool2);
+      cudaFree(doff2);
+    }
   }
   return 0;
 }
