@@ -105,8 +105,9 @@ typedef struct {
                                    regions leave, in whole slabs (aeg_pool_region reports it)   */
   uint64_t device_weight_bytes; /* self-managed weights region (bump allocated)               */
   uint64_t host_kv_bytes;       /* unified CPU KV cache, pinned once at init  */
-  uint64_t dev_slab_bytes;      /* slab size of the device pool          */
-  uint64_t host_slab_bytes;     /* slab size of the host pool                                 */
+  uint64_t dev_slab_bytes;      /* slab size of the device pool; a multiple
+                                   of 16 bytes (INVALID otherwise)                             */
+  uint64_t host_slab_bytes;     /* slab size of the host pool (multiple of 16 bytes)          */
   uint64_t stage_ring_bytes;    /* pinned Stage Buffer for weights (2 GB)      */
   uint64_t stage_chunk_bytes;   /* weight pipeline chunk                                      */
   uint64_t staging_slot_bytes;  /* device staging slot for KV gather/scatter                  */

@@ -5,7 +5,8 @@
 namespace aeg {
 
 void SlabPool::init(int pool_id, uint64_t bytes, uint64_t sbytes, int lay) {
-  AEG_REQUIRE(sbytes > 0, AEG_ERR_INVALID, "slab size must be > 0");
+  AEG_REQUIRE(sbytes > 0 && sbytes % 16 == 0, AEG_ERR_INVALID,
+              "slab size must be a positive multiple of 16 bytes (16-byte vector and bulk copies)");
   AEG_REQUIRE(lay == AEG_LAYER_MAJOR || lay == AEG_BLOCK_MAJOR, AEG_ERR_INVALID, "bad slab layout %d", lay);
   AEG_REQUIRE(bytes / sbytes < (1u << 30), AEG_ERR_INVALID, "too many slabs");
   id = pool_id;

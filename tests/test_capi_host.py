@@ -283,3 +283,12 @@ def test_bench_allocator_leg_runs_on_a_host_only_context():
     r = bench.allocator_leg(aeg, reps=2)
     assert r["per_request_alloc_us_p50"] > 0 and r["batch_alloc_ns_per_block"] > 0
     assert r["batch_free_us"] > 0 and "3970" in r["workload"]
+
+
+def test_slab_size_must_keep_16_byte_alignment():
+    """Every copy is 16-byte vectors or bulk copies: slab bases must stay 16-byte aligned."""
+    for bad in (SLAB + 8, 1000):
+        with pytest.raises(aeg.AegError) as e:
+            aeg.Context(0, aeg.default_config(device_kv_bytes=3 * bad, host_kv_bytes=3 * SLAB, dev_slab_bytes=bad,
+                                              host_slab_bytes=SLAB, flags=aeg.CFG_HOST_ONLY | aeg.CFG_NO_DAEMON))
+        assert e.value.code == aeg.ERR_INVALID
