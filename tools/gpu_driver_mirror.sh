@@ -10,4 +10,4 @@ t0=$(date +%s)
 timeout 600 python bench.py --impl reference --gpus 1 --steps ${REF_STEPS:-20} --warmup ${REF_WARMUP:-5} > gpurun_out/bench_ref.json 2> gpurun_out/bench_ref.err; echo "ref rc=$? $(( $(date +%s)-t0 ))s" >> gpurun_out/bench_ref.err
 t0=$(date +%s)
 timeout 3000 python bench.py --gpus 1 --steps ${STEPS:-20} --warmup ${WARMUP:-5} > gpurun_out/bench.json 2> gpurun_out/bench.err; echo "bench rc=$? $(( $(date +%s)-t0 ))s" >> gpurun_out/bench.err
-tail -3 gpurun_out/gpu_tests.log gpurun_out/smoke.log gpurun_out/bench_ref.err gpurun_out/bench.err
+for f in gpurun_out/gpu_tests.log gpurun_out/smoke.log gpurun_out/bench_ref.err gpurun_out/bench.err; do tail -n 3 $f; done
