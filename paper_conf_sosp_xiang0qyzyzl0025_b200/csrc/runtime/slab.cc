@@ -16,8 +16,7 @@ void SlabPool::init(int pool_id, uint64_t bytes, uint64_t sbytes, int lay) {
   n_slabs = uint32_t(bytes / sbytes);
   slabs_.assign(n_slabs, Slab{});
   shapes_.clear();
-  quarantine_.clear();
-  access_.clear();
+  qlist_.clear();
   used_ = assigned_ = peak_used_ = peak_assigned_ = 0;
 }
 
@@ -60,6 +59,8 @@ void SlabPool::alloc(const Shape& sh, int32_t n, aeg_block* out) {
     sl.shape = sid;
     sl.k = kk;
     sl.st.assign(kk, 0);
+    sl.acc.clear();
+    sl.acc.resize(kk);
     sl.n_owned = sl.n_quar = 0;
     assigned_ += slab_bytes;
   }
@@ -106,18 +107,17 @@ void SlabPool::check_geometry(const aeg_block* b, int32_t n, const Shape& sh) co
                 "peer block 0x%llx outside the peer pool", (unsigned long long)b[i]);
 }
 
-bool SlabPool::busy(aeg_block b, std::vector<uint64_t>* xs) {
-  auto it = access_.find(b);
-  if (it == access_.end()) return false;
+bool SlabPool::busy(aeg_block b, XSet* xs) {
+  const Access& a = acc(b);
   bool any = false;
   auto add = [&](uint64_t x) {
     if (x && !is_done(x)) {
       any = true;
-      if (xs) xs->push_back(x);
+      if (xs) xs->push(x);
     }
   };
-  add(it->second.writer);
-  for (uint64_t r : it->second.readers) add(r);
+  add(a.writer);
+  a.readers.each(add);
   return any;
 }
 
@@ -127,28 +127,32 @@ void SlabPool::maybe_unassign(uint32_t s) {
     sl.shape = -1;
     sl.k = 0;
     sl.st.clear();
+    sl.acc.clear();
     assigned_ -= slab_bytes;
   }
 }
 
 void SlabPool::free(const aeg_block* b, int32_t n) {
   check_owned(b, n, nullptr);
+  uint32_t last = UINT32_MAX;
   std::vector<uint32_t> touched;
   for (int32_t i = 0; i < n; ++i) {
     const uint32_t s = block_slab(b[i]), j = block_idx(b[i]);
     Slab& sl = slabs_[s];
     used_ -= shapes_[sl.shape].block();
     sl.n_owned--;
-    std::vector<uint64_t> xs;
+    Access& a = sl.acc[j];
+    XSet xs;
     if (busy(b[i], &xs)) {
       sl.st[j] = 2;
       sl.n_quar++;
-      quarantine_[b[i]] = std::move(xs);
+      a.quar = std::move(xs);
+      qlist_.push_back(b[i]);
     } else {
       sl.st[j] = 0;
-      access_.erase(b[i]);
+      a = Access{};
     }
-    touched.push_back(s);
+    if (s != last) touched.push_back(last = s);
   }
   for (uint32_t s : touched) maybe_unassign(s);
 }
@@ -164,74 +168,66 @@ void SlabPool::free_after(const aeg_block* b, int32_t n, uint64_t x) {
     Slab& sl = slabs_[s];
     used_ -= shapes_[sl.shape].block();
     sl.n_owned--;
-    std::vector<uint64_t> xs;
+    XSet xs;
     busy(b[i], &xs);
-    xs.push_back(x);
+    xs.push(x);
     sl.st[j] = 2;
     sl.n_quar++;
-    quarantine_[b[i]] = std::move(xs);
+    sl.acc[j].quar = std::move(xs);
+    qlist_.push_back(b[i]);
   }
 }
 
 uint64_t SlabPool::reclaim() {
   uint64_t released = 0;
   std::vector<uint32_t> touched;
-  for (auto it = quarantine_.begin(); it != quarantine_.end();) {
+  for (size_t q = 0; q < qlist_.size();) {
+    const aeg_block blk = qlist_[q];
+    Access& a = acc(blk);
     bool done = true;
-    for (uint64_t x : it->second) done = done && is_done(x);
+    a.quar.each([&](uint64_t x) { done = done && is_done(x); });
     if (!done) {
-      ++it;
+      ++q;
       continue;
     }
-    const uint32_t s = block_slab(it->first), j = block_idx(it->first);
+    const uint32_t s = block_slab(blk), j = block_idx(blk);
     slabs_[s].st[j] = 0;
     slabs_[s].n_quar--;
-    access_.erase(it->first);
+    a = Access{};
     touched.push_back(s);
-    it = quarantine_.erase(it);
+    qlist_[q] = qlist_.back();  // unordered: swap-pop
+    qlist_.pop_back();
     ++released;
   }
+  std::sort(touched.begin(), touched.end());
+  touched.erase(std::unique(touched.begin(), touched.end()), touched.end());
   for (uint32_t s : touched) maybe_unassign(s);
   return released;
 }
 
 void SlabPool::deps_for_read(aeg_block b, std::vector<uint64_t>& deps) {
-  auto it = access_.find(b);
-  if (it != access_.end() && it->second.writer && !is_done(it->second.writer)) deps.push_back(it->second.writer);
+  const Access& a = acc(b);
+  if (a.writer && !is_done(a.writer)) deps.push_back(a.writer);
 }
 
 void SlabPool::deps_for_write(aeg_block b, std::vector<uint64_t>& deps) {
-  auto it = access_.find(b);
-  if (it == access_.end()) return;
-  if (it->second.writer && !is_done(it->second.writer)) deps.push_back(it->second.writer);
-  for (uint64_t r : it->second.readers)
+  const Access& a = acc(b);
+  if (a.writer && !is_done(a.writer)) deps.push_back(a.writer);
+  a.readers.each([&](uint64_t r) {
     if (!is_done(r)) deps.push_back(r);
+  });
 }
 
 void SlabPool::note_read(aeg_block b, uint64_t x) {
-  Access& a = access_[b];
-  auto& r = a.readers;
-  r.erase(std::remove_if(r.begin(), r.end(), [&](uint64_t y) { return is_done(y); }), r.end());
-  r.push_back(x);
+  Access& a = acc(b);
+  a.readers.erase_if([&](uint64_t y) { return is_done(y); });
+  a.readers.push(x);
 }
 
 void SlabPool::note_write(aeg_block b, uint64_t x) {
-  Access& a = access_[b];
+  Access& a = acc(b);
   a.writer = x;
   a.readers.clear();
-}
-
-void SlabPool::forget_completed() {
-  for (auto it = access_.begin(); it != access_.end();) {
-    Access& a = it->second;
-    if (a.writer && is_done(a.writer)) a.writer = 0;
-    a.readers.erase(std::remove_if(a.readers.begin(), a.readers.end(), [&](uint64_t y) { return is_done(y); }),
-                    a.readers.end());
-    if (!a.writer && a.readers.empty() && !quarantine_.count(it->first))
-      it = access_.erase(it);
-    else
-      ++it;
-  }
 }
 
 void SlabPool::stats(aeg_pool_stats* o) const {
