@@ -143,7 +143,10 @@ void Ctx::init(int dev, const aeg_config& c) {
   }
   pool[AEG_POOL_DEVICE].init(AEG_POOL_DEVICE, cfg.device_kv_bytes, cfg.dev_slab_bytes, cfg.dev_slab_layout);
   pool[AEG_POOL_HOST].init(AEG_POOL_HOST, cfg.host_kv_bytes, cfg.host_slab_bytes, cfg.host_slab_layout);
-  for (auto& p : pool) p.is_done = [this](uint64_t x) { return is_done(x); };
+  for (auto& p : pool) {
+    p.is_done = [this](uint64_t x) { return is_done(x); };
+    p.done_below = &done_below;
+  }
   if (host_only) {
     if (!(cfg.flags & AEG_CFG_NO_DAEMON)) daemon = std::thread([this] { daemon_loop(); });
     return;
@@ -340,6 +343,14 @@ bool Ctx::is_done(uint64_t x) {
 }
 
 void Ctx::poll() {
+  poll_events();
+  uint64_t lo = next_xid;  // the lowest id still incomplete bounds the completed prefix
+  for (auto& kv : xfers)
+    if (!kv.second->complete.load(std::memory_order_acquire)) lo = std::min(lo, kv.first);
+  done_below = lo;
+}
+
+void Ctx::poll_events() {
   if (host_only) {
     for (auto& kv : xfers)
       if (kv.second->debug_done) kv.second->complete.store(true);

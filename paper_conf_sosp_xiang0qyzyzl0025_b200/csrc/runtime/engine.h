@@ -164,6 +164,7 @@ struct Ctx {
   TableArena tables;
 
   std::unordered_map<uint64_t, std::unique_ptr<Xfer>> xfers;
+  uint64_t done_below = 1;  // every transfer id below this has completed (updated by poll, under mu)
   uint64_t next_xid = 1;
   std::vector<cudaEvent_t> ev_pool, ev_pool_ipc;
 
@@ -191,7 +192,8 @@ struct Ctx {
 
   // ---- transfers (engine.cc)
   bool is_done(uint64_t x);        // completion observed (or transfer already reaped)
-  void poll();                     // query events of in-flight transfers (caller holds mu)
+  void poll();                     // poll_events + advance done_below (caller holds mu)
+  void poll_events();              // query the completion events of in-flight transfers
   void housekeeping();             // poll + reclaim + release tables + reap (caller holds mu)
   Xfer* new_xfer(int kind, int32_t L, bool ipc);
   Xfer* enqueuing = nullptr;       // transfer whose enqueue is in progress (error recovery)

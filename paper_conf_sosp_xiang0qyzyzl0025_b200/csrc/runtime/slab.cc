@@ -111,7 +111,7 @@ bool SlabPool::busy(aeg_block b, XSet* xs) {
   const Access& a = acc(b);
   bool any = false;
   auto add = [&](uint64_t x) {
-    if (x && !is_done(x)) {
+    if (x && !done(x)) {
       any = true;
       if (xs) xs->push(x);
     }
@@ -184,9 +184,9 @@ uint64_t SlabPool::reclaim() {
   for (size_t q = 0; q < qlist_.size();) {
     const aeg_block blk = qlist_[q];
     Access& a = acc(blk);
-    bool done = true;
-    a.quar.each([&](uint64_t x) { done = done && is_done(x); });
-    if (!done) {
+    bool all = true;
+    a.quar.each([&](uint64_t x) { all = all && done(x); });
+    if (!all) {
       ++q;
       continue;
     }
@@ -205,22 +205,23 @@ uint64_t SlabPool::reclaim() {
   return released;
 }
 
+// (consecutive blocks usually share their last transfer: skip immediate repeats; callers dedupe)
 void SlabPool::deps_for_read(aeg_block b, std::vector<uint64_t>& deps) {
   const Access& a = acc(b);
-  if (a.writer && !is_done(a.writer)) deps.push_back(a.writer);
+  if (a.writer && (deps.empty() || deps.back() != a.writer) && !done(a.writer)) deps.push_back(a.writer);
 }
 
 void SlabPool::deps_for_write(aeg_block b, std::vector<uint64_t>& deps) {
   const Access& a = acc(b);
-  if (a.writer && !is_done(a.writer)) deps.push_back(a.writer);
+  if (a.writer && (deps.empty() || deps.back() != a.writer) && !done(a.writer)) deps.push_back(a.writer);
   a.readers.each([&](uint64_t r) {
-    if (!is_done(r)) deps.push_back(r);
+    if ((deps.empty() || deps.back() != r) && !done(r)) deps.push_back(r);
   });
 }
 
 void SlabPool::note_read(aeg_block b, uint64_t x) {
   Access& a = acc(b);
-  a.readers.erase_if([&](uint64_t y) { return is_done(y); });
+  a.readers.erase_if([&](uint64_t y) { return done(y); });
   a.readers.push(x);
 }
 

@@ -84,6 +84,9 @@ class SlabPool {
   int layout = AEG_LAYER_MAJOR;
   uint32_t n_slabs = 0;
   std::function<bool(uint64_t)> is_done;  // transfer id -> completion observed
+  // Owner-maintained watermark: every transfer id below it has completed (fast path of done()).
+  const uint64_t* done_below = nullptr;
+  bool done(uint64_t x) const { return (done_below && x < *done_below) || is_done(x); }
 
   uint32_t k(const Shape& sh) const { return uint32_t(slab_bytes / sh.block()); }
   // Byte offset (from the pool base) of layer 0 of block b, and the per-layer stride:
