@@ -629,9 +629,12 @@ def c1_leg(aeg, torch, kernel, reps=200):
     lens = gi.request_lengths(1, 8, 1, 256, forced=(1, 16, 17, 255, 256))
     nb = sum(-(-t // 16) for t in lens)
     kib = 1024
+    # staging slots of 8 MiB: the whole 2.3 MiB batch (both layers) is one segment, i.e. one gather /
+    # scatter launch and one copy per host run (1 MiB slots cut each layer in two: 4 segments and
+    # ~2x the enqueue time, tools/enqueue_probe.py)
     ctx = aeg.Context(0, aeg.default_config(device_kv_bytes=32 * 256 * kib, host_kv_bytes=32 * 256 * kib,
                                             dev_slab_bytes=256 * kib, host_slab_bytes=256 * kib,
-                                            staging_slot_bytes=1 << 20, staging_slots=2, stage_ring_bytes=2 << 20,
+                                            staging_slot_bytes=8 << 20, staging_slots=2, stage_ring_bytes=2 << 20,
                                             stage_chunk_bytes=1 << 20, device_weight_bytes=2 << 20,
                                             table_arena_bytes=2 << 20, host_threads=1, kernel=kernel))
     dbase, _ = ctx.pool_region(0)

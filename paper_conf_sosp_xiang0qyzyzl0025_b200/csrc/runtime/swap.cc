@@ -7,6 +7,9 @@
 //   swap-in  : s_h2d    (copy engine)            ->  s_scatter (kernel, high priority)
 // The two halves of a direction hand staging slots back and forth with full/free events.
 #include <algorithm>
+#include <chrono>
+#include <cstdio>
+#include <cstdlib>
 #include <cstring>
 
 #include "engine.h"
@@ -244,14 +247,43 @@ static int impl_of(const aeg_config& cfg, uint64_t chunk) {
   return chunk <= (16u << 10) ? IMPL_BULKW : IMPL_BULK;
 }
 
+// Optional host-side phase timer of swap_out (AEG_HOST_PROFILE=1: totals printed at exit): where
+// the enqueue time of a call goes (validation, rule bookkeeping, table, segments, notes, free).
+namespace {
+struct HostProf {
+  bool on = getenv("AEG_HOST_PROFILE") != nullptr;
+  double t[8] = {0};
+  uint64_t calls = 0;
+  ~HostProf() {
+    if (on && calls)
+      fprintf(stderr, "[aeg host profile] swap_out x%llu, us per call: validate %.1f deps %.1f table %.1f "
+              "plan %.1f segments %.1f record %.1f notes %.1f free %.1f\n", (unsigned long long)calls,
+              t[0] / calls, t[1] / calls, t[2] / calls, t[3] / calls, t[4] / calls, t[5] / calls, t[6] / calls,
+              t[7] / calls);
+  }
+} g_prof;
+struct PhaseClock {
+  std::chrono::steady_clock::time_point t0 = std::chrono::steady_clock::now();
+  void lap(int i) {
+    if (!g_prof.on) return;
+    auto t1 = std::chrono::steady_clock::now();
+    g_prof.t[i] += std::chrono::duration<double, std::micro>(t1 - t0).count();
+    t0 = t1;
+  }
+};
+}  // namespace
+
 // ----------------------------------------------------------------------------- swap-out H3
 uint64_t Ctx::swap_out(const Shape& sh, const aeg_block* dev, const aeg_block* host, int32_t n, uint32_t flags) {
   AEG_REQUIRE(!host_only, AEG_ERR_STATE, "host-only context has no data path");
   SlabPool &dp = pool[AEG_POOL_DEVICE], &hp = pool[AEG_POOL_HOST];
+  PhaseClock pc;
+  if (g_prof.on) g_prof.calls++;
   dp.check_owned(dev, n, &sh);
   hp.check_owned(host, n, &sh);
   AEG_REQUIRE(sh.chunk() <= ring_out.slot_bytes, AEG_ERR_INVALID, "chunk larger than a staging slot");
   Xfer* x = new_xfer(X_SWAP_OUT, sh.L, ipc_events(flags));
+  pc.lap(0);
   std::vector<uint64_t> rdeps, wdeps;
   if (!(flags & AEG_NO_DEPS)) {
     for (int32_t i = 0; i < n; ++i) dp.deps_for_read(dev[i], rdeps);
@@ -259,6 +291,7 @@ uint64_t Ctx::swap_out(const Shape& sh, const aeg_block* dev, const aeg_block* h
   }
   rdeps = uniq(rdeps);
   wdeps = uniq(wdeps);
+  pc.lap(1);
   char *htab = nullptr, *dtab = nullptr;
   if (n > 0) {
     alloc_table(uint64_t(n) * 8, x->id, &htab, &dtab);
@@ -266,6 +299,7 @@ uint64_t Ctx::swap_out(const Shape& sh, const aeg_block* dev, const aeg_block* h
     for (int32_t i = 0; i < n; ++i) t[i] = dp.off0(dev[i], sh);
     fetch_table(dtab, htab, uint64_t(n) * 8, s_gather);
   }
+  pc.lap(2);
   const auto segs = plan(sh.L, n, sh.chunk(), ring_out.slot_bytes);
   const auto runs = runs_of(host, n);
   const uint64_t dstride = dp.lstride(sh);
@@ -286,6 +320,7 @@ uint64_t Ctx::swap_out(const Shape& sh, const aeg_block* dev, const aeg_block* h
   } else {
     x->piece_lo.clear();
   }
+  pc.lap(3);
   int32_t pidx = 0;
   for (const Seg& g : segs) {
     if (g.i0 == 0) pidx = 0;
@@ -336,12 +371,16 @@ uint64_t Ctx::swap_out(const Shape& sh, const aeg_block* dev, const aeg_block* h
     if (g.i1 == n)
       for (int32_t l = g.la; l < g.lb; ++l) record(x, l, s_d2h);
   }
+  pc.lap(4);
   if (n == 0)
     for (int32_t l = 0; l < sh.L; ++l) record(x, l, s_d2h);
   record(x, -1, s_d2h);
+  pc.lap(5);
   for (int32_t i = 0; i < n; ++i) dp.note_read(dev[i], x->id);
   for (int32_t i = 0; i < n; ++i) hp.note_write(host[i], x->id);
+  pc.lap(6);
   if (flags & AEG_FREE_SRC) dp.free(dev, n);
+  pc.lap(7);
   return x->id;
 }
 

@@ -14,10 +14,10 @@ import paper_conf_sosp_xiang0qyzyzl0025_b200 as aeg  # noqa: E402
 
 sht = gi.KV_SHAPES["tiny"]
 KIB = 1024
-for slab_kib in (256, 4096):
+for slab_kib, slot_mib in ((256, 1), (4096, 1), (256, 8)):
     ctx = aeg.Context(0, aeg.default_config(device_kv_bytes=64 * 256 * KIB, host_kv_bytes=64 * slab_kib * KIB,
                                             dev_slab_bytes=256 * KIB, host_slab_bytes=slab_kib * KIB,
-                                            staging_slot_bytes=1 << 20, staging_slots=2, stage_ring_bytes=2 << 20,
+                                            staging_slot_bytes=slot_mib << 20, staging_slots=2, stage_ring_bytes=2 << 20,
                                             stage_chunk_bytes=1 << 20, device_weight_bytes=2 << 20,
                                             table_arena_bytes=2 << 20, host_threads=1))
     for nb in (1, 8, 75):
@@ -41,7 +41,7 @@ for slab_kib in (256, 4096):
                 out.append((t1 - t0) * 1e6)
                 inn.append((t2 - t1) * 1e6)
         runs = -(-nb // ((slab_kib * KIB) // (2 * 32 * KIB)))
-        print(f"host slab {slab_kib:5d} KiB  blocks {nb:3d} (host runs ~{runs:2d}): enqueue swap_out "
+        print(f"slot {slot_mib} MiB host slab {slab_kib:5d} KiB  blocks {nb:3d} (host runs ~{runs:2d}): enqueue swap_out "
               f"{statistics.median(out):6.1f} us, swap_in {statistics.median(inn):6.1f} us", flush=True)
     ctx.shutdown()
 # the CUDA calls themselves, for scale
