@@ -140,9 +140,23 @@ static void host_dmas(const SlabPool& hp, char* hbase, const Shape& sh, const st
                       char* slot, cudaMemcpyKind dir, cudaStream_t s) {
   const uint64_t Cl = sh.chunk(), hstride = hp.lstride(sh);
   const int32_t nseg = g.i1 - g.i0, nl = g.lb - g.la;
-  if (hp.layout == AEG_LAYER_MAJOR && nl == 1) {
-    // One layer: runs of equal length whose host addresses step by a constant pitch (typically whole
-    // slabs: k blocks, pitch S) become ONE 2-D copy — fewer copy-engine commands per layer.
+  if (hp.layout == AEG_LAYER_MAJOR) {
+    // Within one layer, runs of equal length whose host addresses step by a constant pitch
+    // (typically whole slabs: k blocks, pitch S) become ONE 2-D copy.  The grouping is the same in
+    // every layer (layers differ by a constant offset), so a segment costs nl x groups copies this
+    // way, or one copy per run (2-D over its nl layers) the other way: take the fewer commands.
+    struct Group {
+      int32_t a0, m;
+      size_t rows;
+      int64_t pitch;
+      aeg_block first;  // host block of the group's first row at index a0
+    };
+    std::vector<Group> groups;
+    size_t nruns = 0;
+    auto host_of = [&](aeg_block first_of_run, int32_t run_i0, int32_t a, int32_t l) {
+      const aeg_block hb = make_block(AEG_POOL_HOST, block_slab(first_of_run), block_idx(first_of_run) + uint32_t(a - run_i0));
+      return hbase + hp.off0(hb, sh) + uint64_t(l) * hstride;
+    };
     size_t q = 0;
     while (q < runs.size()) {
       const Run& r0 = runs[q];
@@ -151,41 +165,44 @@ static void host_dmas(const SlabPool& hp, char* hbase, const Shape& sh, const st
         ++q;
         continue;
       }
-      auto host_of = [&](const Run& r, int32_t a) {
-        const aeg_block hb = make_block(AEG_POOL_HOST, block_slab(r.first), block_idx(r.first) + uint32_t(a - r.i0));
-        return hbase + hp.off0(hb, sh) + uint64_t(g.la) * hstride;
-      };
-      char* h0 = host_of(r0, a0);
       const int32_t m = b0 - a0;
       size_t e = q + 1;
       int64_t pitch = 0;
-      char* prev = h0;
+      char* prev = host_of(r0.first, r0.i0, a0, g.la);
       while (e < runs.size()) {  // extend while the next run is whole, same length, same pitch
         const Run& r = runs[e];
         if (r.i0 < g.i0 || r.i0 + r.m > g.i1 || r.m != m || r.i0 != a0 + int32_t(e - q) * m) break;
-        char* cur = host_of(r, r.i0);
+        char* cur = host_of(r.first, r.i0, r.i0, g.la);
         const int64_t p = cur - prev;
         if (e == q + 1) pitch = p;
         if (p != pitch || p < int64_t(m) * int64_t(Cl) || p > max_pitch()) break;
         prev = cur;
         ++e;
       }
-      char* st0 = slot + uint64_t(a0 - g.i0) * Cl;
-      const uint64_t w = uint64_t(m) * Cl;
-      const size_t rows = e - q;
-      if (rows == 1) {
-        if (dir == cudaMemcpyDeviceToHost)
-          CUDA_TRY(cudaMemcpyAsync(h0, st0, w, dir, s));
-        else
-          CUDA_TRY(cudaMemcpyAsync(st0, h0, w, dir, s));
-      } else if (dir == cudaMemcpyDeviceToHost) {
-        CUDA_TRY(cudaMemcpy2DAsync(h0, size_t(pitch), st0, w, w, rows, dir, s));
-      } else {
-        CUDA_TRY(cudaMemcpy2DAsync(st0, w, h0, size_t(pitch), w, rows, dir, s));
-      }
+      groups.push_back({a0, m, e - q, pitch,
+                        make_block(AEG_POOL_HOST, block_slab(r0.first), block_idx(r0.first) + uint32_t(a0 - r0.i0))});
+      nruns += e - q;
       q = e;
     }
-    return;
+    if (nl == 1 || uint64_t(nl) * groups.size() < nruns) {
+      for (int32_t t = 0; t < nl; ++t)
+        for (const Group& gr : groups) {
+          char* h0 = hbase + hp.off0(gr.first, sh) + uint64_t(g.la + t) * hstride;
+          char* st0 = slot + (uint64_t(t) * nseg + uint64_t(gr.a0 - g.i0)) * Cl;
+          const uint64_t w = uint64_t(gr.m) * Cl;
+          if (gr.rows == 1) {
+            if (dir == cudaMemcpyDeviceToHost)
+              CUDA_TRY(cudaMemcpyAsync(h0, st0, w, dir, s));
+            else
+              CUDA_TRY(cudaMemcpyAsync(st0, h0, w, dir, s));
+          } else if (dir == cudaMemcpyDeviceToHost) {
+            CUDA_TRY(cudaMemcpy2DAsync(h0, size_t(gr.pitch), st0, w, w, gr.rows, dir, s));
+          } else {
+            CUDA_TRY(cudaMemcpy2DAsync(st0, w, h0, size_t(gr.pitch), w, gr.rows, dir, s));
+          }
+        }
+      return;
+    }
   }
   for (const Run& r : runs) {
     const int32_t a = std::max(r.i0, g.i0), b = std::min(r.i0 + r.m, g.i1);
