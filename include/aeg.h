@@ -67,9 +67,12 @@ enum {
   AEG_FREE_SRC = 1u << 0,  /* free the source blocks once enqueued; they sit in the move list
                               until the transfer completes               */
   AEG_NO_DEPS = 1u << 1,   /* caller guarantees ordering: skip last-writer stream waits (❷❸) */
-  AEG_IPC_EVENTS = 1u << 2 /* interprocess-capable events, so aeg_xfer_export works across
+  AEG_IPC_EVENTS = 1u << 2, /* interprocess-capable events, so aeg_xfer_export works across
                               processes (implied for AEG_CFG_SHARED_HOST contexts, for
                               aeg_kv_swap_in_from a peer and for migrates to another process)  */
+  AEG_MIGRATE_CE = 1u << 3  /* aeg_kv_migrate only: the copy-engine route instead of the fused
+                              kernel — gather kernel into the out staging ring, then copy-engine
+                              commands into the destination pool (zero SMs on the link)         */
 };
 /* weight split kinds (Megatron-style tensor parallelism, reading 18) */
 enum { AEG_SPLIT_REPLICATED = 0, AEG_SPLIT_COL = 1, AEG_SPLIT_ROW = 2, AEG_SPLIT_VOCAB = 3 };
@@ -252,7 +255,11 @@ int aeg_kv_swap_in(aeg_ctx ctx, const aeg_kv_shape* shape, const aeg_block* host
  * aeg_import_peer, or -1 for this context's own device pool (local relocation).  dst handles are
  * allocated by the peer in its device pool and are trusted (validated against the peer's
  * geometry only).  Per-layer events are interprocess-capable; export them with aeg_xfer_export.
- * AEG_FREE_SRC frees the source blocks. */
+ * AEG_FREE_SRC frees the source blocks.  AEG_MIGRATE_CE takes the copy-engine route (SURVEY H5
+ * alternative): per staging segment a gather kernel packs the source blocks into the out staging
+ * ring, then copy engines write the destination runs (one command per run and layer, or one 2-D
+ * command per layer across equal whole runs); the decode GPU's SMs are never used and the source
+ * GPU's only for the HBM-speed gather.  Same bytes, same events, same rules. */
 int aeg_kv_migrate(aeg_ctx ctx, const aeg_kv_shape* shape, const aeg_block* src, int32_t peer,
                    const aeg_block* dst, int32_t n, uint32_t flags, aeg_xfer* out);
 

@@ -23,7 +23,7 @@ POOL_DEVICE, POOL_HOST = 0, 1
 LAYER_MAJOR, BLOCK_MAJOR = 0, 1
 OK, NOT_READY, ERR_INVALID, ERR_OOM, ERR_CUDA, ERR_STATE = 0, 1, -1, -2, -3, -4
 READY_QUERY, READY_WAIT_STREAM, READY_BLOCK = 0, 1, 2
-FREE_SRC, NO_DEPS = 1, 2
+FREE_SRC, NO_DEPS, IPC_EVENTS, MIGRATE_CE = 1, 2, 4, 8
 SPLIT_REPLICATED, SPLIT_COL, SPLIT_ROW, SPLIT_VOCAB = 0, 1, 2, 3
 CFG_HOST_ONLY, CFG_NO_DAEMON, CFG_TIMING, CFG_SHARED_HOST = 1, 2, 4, 8
 KERNEL_AUTO, KERNEL_LSU, KERNEL_BULK, KERNEL_WARP, KERNEL_BULKW = 0, 1, 2, 3, 4

@@ -217,6 +217,7 @@ void Ctx::init(int dev, const aeg_config& c) {
   CUDA_TRY(cudaStreamCreateWithFlags(&s_d2h, cudaStreamNonBlocking));
   CUDA_TRY(cudaStreamCreateWithFlags(&s_h2d, cudaStreamNonBlocking));
   CUDA_TRY(cudaStreamCreateWithFlags(&s_weights, cudaStreamNonBlocking));
+  CUDA_TRY(cudaStreamCreateWithFlags(&s_p2p, cudaStreamNonBlocking));
   CUDA_TRY(cudaEventCreateWithFlags(&fence_ev, cudaEventDisableTiming));
   for (Ring* r : {&ring_out, &ring_in}) {
     r->slot_bytes = cfg.staging_slot_bytes;
@@ -230,7 +231,7 @@ void Ctx::shutdown() {
   if (!host_only) {
     weights_stop();
     cudaSetDevice(device);
-    for (cudaStream_t s : {s_gather, s_d2h, s_h2d, s_scatter, s_weights, s_migrate})
+    for (cudaStream_t s : {s_gather, s_d2h, s_h2d, s_scatter, s_weights, s_migrate, s_p2p})
       if (s) cudaStreamSynchronize(s);
   }
   {
@@ -271,7 +272,7 @@ void Ctx::shutdown() {
   }
   for (auto& r : registered) cudaHostUnregister(r.first);
   cudaEventDestroy(fence_ev);
-  for (cudaStream_t s : {s_gather, s_d2h, s_h2d, s_scatter, s_weights, s_migrate})
+  for (cudaStream_t s : {s_gather, s_d2h, s_h2d, s_scatter, s_weights, s_migrate, s_p2p})
     if (s) cudaStreamDestroy(s);
   if (dev_mem) cudaFree(dev_mem);
   if (host_mem) unpin_host(host_mem, host_mem_bytes);
@@ -463,7 +464,7 @@ void Ctx::abort_enqueue() {
   Xfer* x = enqueuing;
   enqueuing = nullptr;
   if (!x || host_only) return;
-  for (cudaStream_t s : {s_gather, s_d2h, s_h2d, s_scatter, s_migrate}) cudaStreamSynchronize(s);
+  for (cudaStream_t s : {s_gather, s_d2h, s_h2d, s_scatter, s_migrate, s_p2p}) cudaStreamSynchronize(s);
   (void)cudaGetLastError();
   std::fill(x->recorded.begin(), x->recorded.end(), uint8_t(1));
   x->done_recorded = true;
@@ -658,6 +659,7 @@ std::string Ctx::sname(cudaStream_t s) const {
   if (s == s_scatter) return "scatter";
   if (s == s_weights) return "weights";
   if (s == s_migrate) return "migrate";
+  if (s == s_p2p) return "p2p";
   char b[32];
   snprintf(b, sizeof b, "u%p", (void*)s);
   return b;

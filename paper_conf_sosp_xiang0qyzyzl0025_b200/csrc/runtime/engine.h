@@ -159,6 +159,7 @@ struct Ctx {
 
   cudaStream_t s_gather = nullptr, s_d2h = nullptr, s_h2d = nullptr, s_scatter = nullptr;
   cudaStream_t s_weights = nullptr, s_migrate = nullptr;
+  cudaStream_t s_p2p = nullptr;  // copy-engine hand-off route (AEG_MIGRATE_CE): staging -> peer pool
   cudaEvent_t fence_ev = nullptr;
   Ring ring_out, ring_in;
   TableArena tables;

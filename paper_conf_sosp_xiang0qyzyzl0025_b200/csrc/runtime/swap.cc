@@ -136,8 +136,11 @@ static int64_t max_pitch() {
 
 // Copy-engine DMAs between a staging slot and the host blocks of segment g (layer-major staging
 // image inside the slot).  dir = cudaMemcpyDeviceToHost (swap-out) or HostToDevice (swap-in).
+// `hp` / `hbase` is the pool on the far side of the copy engine: this context's host pool (D2H / H2D)
+// or, for the copy-engine hand-off route, a device pool (this one's or a peer's; kind = Default).
+// to_pool: staging -> pool (swap-out, hand-off) or pool -> staging (swap-in).
 static void host_dmas(const SlabPool& hp, char* hbase, const Shape& sh, const std::vector<Run>& runs, const Seg& g,
-                      char* slot, cudaMemcpyKind dir, cudaStream_t s) {
+                      char* slot, bool to_pool, cudaMemcpyKind dir, cudaStream_t s) {
   const uint64_t Cl = sh.chunk(), hstride = hp.lstride(sh);
   const int32_t nseg = g.i1 - g.i0, nl = g.lb - g.la;
   if (hp.layout == AEG_LAYER_MAJOR) {
@@ -191,11 +194,11 @@ static void host_dmas(const SlabPool& hp, char* hbase, const Shape& sh, const st
           char* st0 = slot + (uint64_t(t) * nseg + uint64_t(gr.a0 - g.i0)) * Cl;
           const uint64_t w = uint64_t(gr.m) * Cl;
           if (gr.rows == 1) {
-            if (dir == cudaMemcpyDeviceToHost)
+            if (to_pool)
               CUDA_TRY(cudaMemcpyAsync(h0, st0, w, dir, s));
             else
               CUDA_TRY(cudaMemcpyAsync(st0, h0, w, dir, s));
-          } else if (dir == cudaMemcpyDeviceToHost) {
+          } else if (to_pool) {
             CUDA_TRY(cudaMemcpy2DAsync(h0, size_t(gr.pitch), st0, w, w, gr.rows, dir, s));
           } else {
             CUDA_TRY(cudaMemcpy2DAsync(st0, w, h0, size_t(gr.pitch), w, gr.rows, dir, s));
@@ -219,12 +222,12 @@ static void host_dmas(const SlabPool& hp, char* hbase, const Shape& sh, const st
         for (int32_t t = 0; t < nl; ++t) {
           char* h = host0 + uint64_t(t) * hstride;
           char* st = st0 + uint64_t(t) * st_pitch;
-          if (dir == cudaMemcpyDeviceToHost)
+          if (to_pool)
             CUDA_TRY(cudaMemcpyAsync(h, st, w, dir, s));
           else
             CUDA_TRY(cudaMemcpyAsync(st, h, w, dir, s));
         }
-      } else if (dir == cudaMemcpyDeviceToHost) {
+      } else if (to_pool) {
         CUDA_TRY(cudaMemcpy2DAsync(host0, hstride, st0, st_pitch, w, nl, dir, s));
       } else {
         CUDA_TRY(cudaMemcpy2DAsync(st0, st_pitch, host0, hstride, w, nl, dir, s));
@@ -234,7 +237,7 @@ static void host_dmas(const SlabPool& hp, char* hbase, const Shape& sh, const st
       for (int32_t t = 0; t < nl; ++t) {
         char* h = host0 + uint64_t(t) * hstride;
         char* st = st0 + uint64_t(t) * st_pitch;
-        if (dir == cudaMemcpyDeviceToHost)
+        if (to_pool)
           CUDA_TRY(cudaMemcpy2DAsync(h, sh.block(), st, Cl, Cl, m, dir, s));
         else
           CUDA_TRY(cudaMemcpy2DAsync(st, Cl, h, sh.block(), Cl, m, dir, s));
@@ -370,7 +373,7 @@ uint64_t Ctx::swap_out(const Shape& sh, const aeg_block* dev, const aeg_block* h
       for (auto& pc : pieces_of(g, sh.chunk(), piece_bytes, runs)) {
         const Seg sub{g.la, g.lb, pc.first, pc.second};
         const uint64_t po = uint64_t(pc.first - g.i0) * sh.chunk();
-        host_dmas(hp, host_kv, sh, runs, sub, sp + po, cudaMemcpyDeviceToHost, s_d2h);
+        host_dmas(hp, host_kv, sh, runs, sub, sp + po, true, cudaMemcpyDeviceToHost, s_d2h);
         if (tracing)
           tr("op d2h d2h r=" + ring_cells("SO", roff + po, uint64_t(pc.second - pc.first) * sh.chunk()) +
              " w=" + cells(1, hp, host, n, g.la, g.lb, pc.first, pc.second));
@@ -379,7 +382,7 @@ uint64_t Ctx::swap_out(const Shape& sh, const aeg_block* dev, const aeg_block* h
         tr_record(s_d2h, pe);
       }
     } else {
-      host_dmas(hp, host_kv, sh, runs, g, sp, cudaMemcpyDeviceToHost, s_d2h);
+      host_dmas(hp, host_kv, sh, runs, g, sp, true, cudaMemcpyDeviceToHost, s_d2h);
       if (tracing)
         tr("op d2h d2h r=" + ring_cells("SO", roff, seg_bytes) + " w=" + cells(1, hp, host, n, g.la, g.lb, g.i0, g.i1));
     }
@@ -535,13 +538,13 @@ uint64_t Ctx::swap_in_from(const Shape& sh, int32_t peer, const aeg_block* host,
         ++pidx;
         const Seg sub{g.la, g.lb, pc.first, pc.second};
         const uint64_t po = uint64_t(pc.first - g.i0) * sh.chunk();
-        host_dmas(hp, hbase, sh, runs, sub, sp + po, cudaMemcpyHostToDevice, s_h2d);
+        host_dmas(hp, hbase, sh, runs, sub, sp + po, false, cudaMemcpyHostToDevice, s_h2d);
         if (tracing)
           tr("op h2d h2d r=" + cells(1, hp, host, n, g.la, g.lb, pc.first, pc.second) + " w=" +
              ring_cells("SI", roff + po, uint64_t(pc.second - pc.first) * sh.chunk()));
       }
     } else {
-      host_dmas(hp, hbase, sh, runs, g, sp, cudaMemcpyHostToDevice, s_h2d);
+      host_dmas(hp, hbase, sh, runs, g, sp, false, cudaMemcpyHostToDevice, s_h2d);
       if (tracing)
         tr("op h2d h2d r=" + cells(1, hp, host, n, g.la, g.lb, g.i0, g.i1) + " w=" + ring_cells("SI", roff, seg_bytes));
     }
@@ -614,12 +617,69 @@ uint64_t Ctx::migrate(const Shape& sh, const aeg_block* src, int32_t peer, const
   for (uint64_t d : wdeps) rdeps.push_back(d);
   rdeps = uniq(rdeps);
   char *htab = nullptr, *dtab = nullptr;
-  if (n > 0) {
+  if (n > 0 && !(flags & AEG_MIGRATE_CE)) {
     alloc_table(uint64_t(n) * 16, x->id, &htab, &dtab);
     uint64_t* t = reinterpret_cast<uint64_t*>(htab);
     for (int32_t i = 0; i < n; ++i) t[i] = dp.off0(src[i], sh);
     for (int32_t i = 0; i < n; ++i) t[n + i] = dg->off0(dst[i], sh);
     fetch_table(dtab, htab, uint64_t(n) * 16, s_migrate);
+  }
+  if (flags & AEG_MIGRATE_CE) {
+    // Copy-engine route (SURVEY H5 alternative; zero SMs on the link): per segment of the out
+    // staging ring, the gather kernel packs the source blocks (HBM), then copy engines move the
+    // segment into the destination pool — one command per destination run and layer, or one 2-D
+    // command per layer across equal whole runs (host_dmas) — on s_p2p; per-layer events there.
+    if (n > 0) {
+      alloc_table(uint64_t(n) * 8, x->id, &htab, &dtab);
+      uint64_t* t = reinterpret_cast<uint64_t*>(htab);
+      for (int32_t i = 0; i < n; ++i) t[i] = dp.off0(src[i], sh);
+      fetch_table(dtab, htab, uint64_t(n) * 8, s_gather);
+    }
+    AEG_REQUIRE(sh.chunk() <= ring_out.slot_bytes, AEG_ERR_INVALID, "chunk larger than a staging slot");
+    const auto segs = plan(sh.L, n, sh.chunk(), ring_out.slot_bytes);
+    const auto runs = runs_of(dst, n);
+    const uint64_t sstride = dp.lstride(sh);
+    for (const Seg& g : segs) {
+      if (g.i0 == 0) wait_deps(s_gather, rdeps, g.la, g.lb);  // rules ❷ (sources) and ❸ (local dst)
+      cudaEvent_t full, freed;
+      uint64_t roff;
+      std::vector<cudaEvent_t> waited;
+      const uint64_t seg_bytes = uint64_t(g.lb - g.la) * uint64_t(g.i1 - g.i0) * sh.chunk();
+      char* sp = ring_out.acquire(seg_bytes, s_gather, &full, &freed, &roff, tracing ? &waited : nullptr);
+      for (cudaEvent_t e : waited) tr_wait(s_gather, e);
+      CopyArgs a;
+      a.src = dev_kv;
+      a.src_off = reinterpret_cast<const uint64_t*>(dtab) + g.i0;
+      a.src_lstride = sstride;
+      a.l_first = g.la;
+      a.dst = sp;
+      a.chunk = sh.chunk();
+      a.nl = g.lb - g.la;
+      a.n = g.i1 - g.i0;
+      launch(0, a, s_gather, impl_of(cfg, sh.chunk()), 0);
+      if (tracing)
+        tr("op gather gather r=" + cells(0, dp, src, n, g.la, g.lb, g.i0, g.i1) + " w=" + ring_cells("SO", roff, seg_bytes));
+      CUDA_TRY(cudaEventRecord(full, s_gather));
+      tr_record(s_gather, full);
+      CUDA_TRY(cudaStreamWaitEvent(s_p2p, full, 0));
+      tr_wait(s_p2p, full);
+      host_dmas(*dg, dbase, sh, runs, g, sp, true, cudaMemcpyDefault, s_p2p);
+      if (tracing)
+        tr("op p2p p2p r=" + ring_cells("SO", roff, seg_bytes) + " w=" +
+           cells(peer < 0 ? 0 : 2, *dg, dst, n, g.la, g.lb, g.i0, g.i1));
+      CUDA_TRY(cudaEventRecord(freed, s_p2p));
+      tr_record(s_p2p, freed);
+      if (g.i1 == n)
+        for (int32_t l = g.la; l < g.lb; ++l) record(x, l, s_p2p);
+    }
+    if (n == 0)
+      for (int32_t l = 0; l < sh.L; ++l) record(x, l, s_p2p);
+    record(x, -1, s_p2p);
+    for (int32_t i = 0; i < n; ++i) dp.note_read(src[i], x->id);
+    if (peer < 0)
+      for (int32_t i = 0; i < n; ++i) dp.note_write(dst[i], x->id);
+    if (flags & AEG_FREE_SRC) dp.free(src, n);
+    return x->id;
   }
   // Layers per launch: every launch pays a fixed ~8-36 us, so pack layers up to a
   // target payload.  Same-device destinations copy at HBM speed (a 133 MiB layer is ~45 us): pack to

@@ -29,8 +29,11 @@ def make(layout, slab=MIB, nslabs=8, kernel=aeg.KERNEL_LSU):
     return ctx, Side(ctx, aeg.POOL_DEVICE, cfg.device_kv_bytes, slab, layout)
 
 
+@pytest.mark.parametrize("ce", [False, True], ids=["kernel", "ce"])
 @pytest.mark.parametrize("kernel", [aeg.KERNEL_LSU, aeg.KERNEL_BULK, aeg.KERNEL_BULKW])
-def test_local_migrate(kernel):
+def test_local_migrate(kernel, ce):
+    """Local relocation (peer -1) through the fused kernel or the copy-engine route (AEG_MIGRATE_CE:
+    gather kernel `kernel` into staging, then copy-engine commands into the destination blocks)."""
     require_gpu()
     ctx, dev = make(aeg.BLOCK_MAJOR, kernel=kernel)
     try:
@@ -40,7 +43,7 @@ def test_local_migrate(kernel):
         fill_blocks(dev, img, SH, so, [(0, j) for j in range(37)])
         dc, do = dev.alloc(SH, 37)
         poison_blocks(dev, img, SH, do)
-        x = ctx.kv_migrate(SH.as_tuple(), sc, -1, dc)
+        x = ctx.kv_migrate(SH.as_tuple(), sc, -1, dc, flags=aeg.MIGRATE_CE if ce else 0)
         exp = OK.migrate(img, dev.geom, img, dev.geom, SH, so, do)
         ctx.layer_ready(x, -1, aeg.READY_BLOCK)
         assert first_diff(dev.read(), exp) is None
@@ -71,7 +74,8 @@ def test_local_migrate_under_an_sm_budget(ctas):
         ctx.shutdown()
 
 
-def test_same_process_peer_migrate_and_imported_events():
+@pytest.mark.parametrize("ce", [False, True], ids=["kernel", "ce"])
+def test_same_process_peer_migrate_and_imported_events(ce):
     require_gpu()
     a, A = make(aeg.LAYER_MAJOR, slab=MIB)
     b, B = make(aeg.BLOCK_MAJOR, slab=MIB + 64 * 1024, nslabs=6)
@@ -85,7 +89,7 @@ def test_same_process_peer_migrate_and_imported_events():
         poison_blocks(B, bimg, SH, do)
         a.import_peer(5, b.export_ipc())
         b.import_peer(0, a.export_ipc())
-        x = a.kv_migrate(SH.as_tuple(), sc, 5, dc)
+        x = a.kv_migrate(SH.as_tuple(), sc, 5, dc, flags=aeg.MIGRATE_CE if ce else 0)
         xi = b.xfer_import(0, a.xfer_export(x))
         for l in range(SH.L):
             b.layer_ready(xi, l, aeg.READY_BLOCK)
@@ -164,7 +168,8 @@ def _decode_body(conn):
     ctx.shutdown()
 
 
-def test_two_process_ipc_migrate():
+@pytest.mark.parametrize("ce", [False, True], ids=["kernel", "ce"])
+def test_two_process_ipc_migrate(ce):
     require_gpu()
     ctxm = mp.get_context("spawn")
     parent, child = ctxm.Pipe()
@@ -187,7 +192,8 @@ def test_two_process_ipc_migrate():
         fill_blocks(A, aimg, SH, so, [(7, j) for j in range(20)])
         blob, dc, do = recv()
         a.import_peer(0, blob)
-        x = a.kv_migrate(SH.as_tuple(), sc, 0, np.array(dc, dtype=np.uint64), flags=aeg.FREE_SRC)
+        x = a.kv_migrate(SH.as_tuple(), sc, 0, np.array(dc, dtype=np.uint64),
+                         flags=aeg.FREE_SRC | (aeg.MIGRATE_CE if ce else 0))
         parent.send(a.xfer_export(x))
         got = np.frombuffer(recv(), dtype=np.uint8)
         geom = OK.PoolGeom(4 * MIB, MIB, aeg.BLOCK_MAJOR)
@@ -327,7 +333,8 @@ def test_two_process_host_route_p_c_d(nblocks):
     assert p.exitcode == 0
 
 
-def test_two_device_same_process_migrate():
+@pytest.mark.parametrize("ce", [False, True], ids=["kernel", "ce"])
+def test_two_device_same_process_migrate(ce):
     """H5 across two GPUs of one process (aeg_import_peer's same-process cross-device branch: peer
     access enabled, the migrate kernel on cuda:0 stores into cuda:1's pool over NVLink): the
     destination image equals oracle.kv.migrate (O7).  Needs two visible GPUs."""
@@ -355,7 +362,7 @@ def test_two_device_same_process_migrate():
         sc, so = A.alloc(SH, 50)
         fill_blocks(A, aimg, SH, so, [(4, j) for j in range(50)])
         a.import_peer(1, b.export_ipc())
-        x = a.kv_migrate(SH.as_tuple(), sc, 1, dc)
+        x = a.kv_migrate(SH.as_tuple(), sc, 1, dc, flags=aeg.MIGRATE_CE if ce else 0)
         a.layer_ready(x, -1, aeg.READY_BLOCK)
         exp = OK.migrate(aimg, A.geom, bimg, B.geom, SH, so, do)
         torch.cuda.set_device(1)

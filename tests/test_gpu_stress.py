@@ -1,5 +1,5 @@
 """Race stress (SURVEY.md §4 race tests; rules ❶❷❸): seeded random sequences of
-swap-out / swap-in / local migrate / free (with FREE_SRC move lists) over small pools, while gate
+swap-out / swap-in / local migrate (fused kernel or copy-engine route) / free (with FREE_SRC move lists) over small pools, while gate
 kernels hold some transfers back and open at random later points, so transfers overlap in every
 order the rules allow.  Checks: (1) the library's own primitive log passes the oracle's
 happens-before checker (oracle/rules.py), including consumer reads after per-layer waits (❶);
@@ -118,7 +118,9 @@ def _stress(seed, cfg, SH, nmax, lo=1):
                     o[:] = ["dev", dc, x]
                 elif op == "mig" and o[0] == "dev":
                     dc = ctx.kv_alloc(0, SH.as_tuple(), len(o[1]))
-                    x = ctx.kv_migrate(SH.as_tuple(), o[1], -1, dc, flags=aeg.FREE_SRC)
+                    # the fused kernel or the copy-engine route (AEG_MIGRATE_CE), at random
+                    ce = aeg.MIGRATE_CE if r.random() < 0.5 else 0
+                    x = ctx.kv_migrate(SH.as_tuple(), o[1], -1, dc, flags=aeg.FREE_SRC | ce)
                     dimg = OK.migrate(dimg, dev.geom, dimg, dev.geom, SH, dec(o[1]), dec(dc))
                     o[:] = ["dev", dc, x]
                 elif op == "free":
