@@ -93,6 +93,13 @@ def _stress(seed, cfg, SH, nmax, lo=1):
                         offs.append(o)
                         keys.append(gi.kv_key(2, step, j, l))
                         dimg[o:o + SH.chunk_bytes()] = gi.region_bytes(SEED, keys[-1], SH.chunk_bytes())
+                # the test's own consumer may still be reading blocks it freed earlier (the library
+                # cannot see reads outside it): like an engine that reuses memory only after its
+                # decode step, drain the consumer stream before the host writes fresh blocks
+                cons.synchronize()
+                flush()
+                log.append(("record", "u0x%x" % cons.cuda_stream, f"cons{step}"))
+                log.append(("sync", f"cons{step}"))
                 D.fill_chunks(dev.base, offs, keys, SH.chunk_bytes(), SEED)
                 # fresh blocks are touched by no incomplete transfer (❸); log the fill as a write
                 flush()
