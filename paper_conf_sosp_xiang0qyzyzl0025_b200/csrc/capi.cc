@@ -350,7 +350,7 @@ int aeg_stream_fence(aeg_ctx ctx, void* stream) {
     cudaStream_t s = static_cast<cudaStream_t>(stream);
     CUDA_TRY(cudaEventRecord(c.fence_ev, s));
     c.tr_record(s, c.fence_ev);
-    for (cudaStream_t t : {c.s_gather, c.s_d2h, c.s_h2d, c.s_scatter, c.s_weights, c.s_migrate}) {
+    for (cudaStream_t t : {c.s_gather, c.s_d2h, c.s_h2d, c.s_scatter, c.s_weights, c.s_migrate, c.s_p2p}) {
       CUDA_TRY(cudaStreamWaitEvent(t, c.fence_ev, 0));
       c.tr_wait(t, c.fence_ev);
     }

@@ -77,6 +77,7 @@ def _stress(seed, cfg, SH, nmax, lo=1):
         objs = []        # [where, handles]
         n_out = 0
         gates = []       # open gates
+        used = [False]   # a consumer read since the consumer stream was last drained
         cons = torch.cuda.Stream()
         for step in range(45):
             op = r.choice(["new", "new", "out", "out", "in", "in", "mig", "free", "gate", "open", "use"])
@@ -93,13 +94,19 @@ def _stress(seed, cfg, SH, nmax, lo=1):
                         offs.append(o)
                         keys.append(gi.kv_key(2, step, j, l))
                         dimg[o:o + SH.chunk_bytes()] = gi.region_bytes(SEED, keys[-1], SH.chunk_bytes())
-                # the test's own consumer may still be reading blocks it freed earlier (the library
-                # cannot see reads outside it): like an engine that reuses memory only after its
-                # decode step, drain the consumer stream before the host writes fresh blocks
-                cons.synchronize()
-                flush()
-                log.append(("record", "u0x%x" % cons.cuda_stream, f"cons{step}"))
-                log.append(("sync", f"cons{step}"))
+                if used[0]:
+                    # the test's own consumer may still be reading blocks freed since (the library
+                    # cannot see reads outside it): like an engine that reuses memory only after its
+                    # decode step, drain the consumer before the host writes fresh blocks — opening
+                    # the gates first, since the consumer may wait on transfers they hold back
+                    for g in gates:
+                        g.open()
+                    gates.clear()
+                    cons.synchronize()
+                    flush()
+                    log.append(("record", "u0x%x" % cons.cuda_stream, f"cons{step}"))
+                    log.append(("sync", f"cons{step}"))
+                    used[0] = False
                 D.fill_chunks(dev.base, offs, keys, SH.chunk_bytes(), SEED)
                 # fresh blocks are touched by no incomplete transfer (❸); log the fill as a write
                 flush()
@@ -148,6 +155,7 @@ def _stress(seed, cfg, SH, nmax, lo=1):
                     flush()
                     log.append(("use", "u0x%x" % cons.cuda_stream,
                                 [f"D:{s}:{j}:{l}" for s, j in dec(o[1]) for l in range(SH.L)]))
+                    used[0] = True
             except aeg.AegError as e:
                 assert e.code == aeg.ERR_OOM, e       # pools are small: OOM is the only legal refusal
             flush()
