@@ -986,7 +986,7 @@ def migrate_leg(aeg, torch, kernel, n_req=16, src_layout=None, dst_layout=None):
     D.fill_chunks(abase, offs, keys, sh.chunk_bytes(), seed)
     a.import_peer(1, b.export_ipc())
 
-    def timed(reps):
+    def timed(reps, flags=0):
         out = []
         for it in range(reps + 2):
             a.kernel_stats_reset()
@@ -994,7 +994,7 @@ def migrate_leg(aeg, torch, kernel, n_req=16, src_layout=None, dst_layout=None):
             e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
             e0.record(s)
             a.stream_fence(s.cuda_stream)
-            x = a.kv_migrate(sht, sc, 1, dc)
+            x = a.kv_migrate(sht, sc, 1, dc, flags=flags)
             a.layer_ready(x, -1, aeg.READY_WAIT_STREAM, s.cuda_stream)
             e1.record(s)
             e1.synchronize()
@@ -1009,9 +1009,12 @@ def migrate_leg(aeg, torch, kernel, n_req=16, src_layout=None, dst_layout=None):
         a.set_migrate_ctas(ctas)
         sweep[ctas] = round(n * sh.block_bytes() / (min(timed(2)) * 1e6), 1)
     a.set_migrate_ctas(0)
+    ce_ms = min(timed(2, aeg.MIGRATE_CE))   # copy-engine route: gather kernel + CE D2D commands
+    doffs = chunk_offsets(b, 0, sht, dc)
+    bad_ce, _ = D.verify_chunks(bbase, doffs, keys, sh.chunk_bytes(), seed)
+    D.fill_chunks(bbase, doffs, [gi.poison_key(gi.TAG_DST, int(o)) for o in doffs], sh.chunk_bytes(), seed)
     times = timed(4)
     nl, nbytes, kms = a.kernel_stats(aeg.K_MIGRATE)
-    doffs = chunk_offsets(b, 0, sht, dc)
     bad, _ = D.verify_chunks(bbase, doffs, keys, sh.chunk_bytes(), seed)
     # baseline on the same blocks: one cudaMemcpyAsync (copy engine, D2D) per (block, layer) chunk
     s = new_stream(torch)
@@ -1033,6 +1036,7 @@ def migrate_leg(aeg, torch, kernel, n_req=16, src_layout=None, dst_layout=None):
             "hbm_GBps": round(2 * payload / (ms * 1e6), 1), "kernel_launches_per_xfer": nl,
             "kernel_ms_per_xfer": round(kms, 3), "bit_exact": bad == 0,
             "GBps_payload_by_ctas": sweep,
+            "ce_route_GBps_payload": round(payload / (ce_ms * 1e6), 1), "ce_route_bit_exact": bad_ce == 0,
             "per_chunk_memcpy_baseline_GBps_payload": round(payload / (min(bt) * 1e6), 1),
             "per_chunk_memcpy_calls": int(len(offs))}
 
@@ -1070,13 +1074,13 @@ def migrate_leg_two_device(aeg, torch, kernel, n_req=16):
         a.import_peer(1, b.export_ipc())
         s = torch.cuda.Stream(device=0)
 
-        def timed(reps):
+        def timed(reps, flags=0):
             out = []
             for it in range(reps + 1):
                 e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
                 e0.record(s)
                 a.stream_fence(s.cuda_stream)
-                x = a.kv_migrate(sht, sc, 1, dc)
+                x = a.kv_migrate(sht, sc, 1, dc, flags=flags)
                 a.layer_ready(x, -1, aeg.READY_WAIT_STREAM, s.cuda_stream)
                 e1.record(s)
                 e1.synchronize()
@@ -1090,6 +1094,7 @@ def migrate_leg_two_device(aeg, torch, kernel, n_req=16):
             a.set_migrate_ctas(ctas)
             sweep[ctas] = round(payload / (min(timed(2)) * 1e6), 1)
         a.set_migrate_ctas(0)
+        ce_ms = min(timed(2, aeg.MIGRATE_CE))
         ms = statistics.median(timed(4))
         torch.cuda.set_device(1)
         bad, _ = D.verify_chunks(bbase, chunk_offsets(b, 0, sht, dc), keys, sh.chunk_bytes(), seed)
@@ -1099,7 +1104,9 @@ def migrate_leg_two_device(aeg, torch, kernel, n_req=16):
                             "one process (direct peer mapping, NVLink)",
                 "payload_bytes": payload, "ms": round(ms, 3), "GBps": round(payload / (ms * 1e6), 1),
                 "frac_of_nvlink_nominal": round(payload / (ms * 1e6) / NVLINK_NOMINAL, 3),
-                "GBps_by_ctas": sweep, "ctas_for_70pct_nvlink": ok[0] if ok else None, "bit_exact": bad == 0}
+                "GBps_by_ctas": sweep, "ctas_for_70pct_nvlink": ok[0] if ok else None, "bit_exact": bad == 0,
+                "ce_route_GBps": round(payload / (ce_ms * 1e6), 1),
+                "ce_route_frac_of_measured_peer_copy": round(payload / (ce_ms * 1e6) / NVLINK_PEER_COPY, 3)}
     finally:
         torch.cuda.set_device(0)
         a.shutdown()
@@ -1212,6 +1219,38 @@ def migrate_leg_dist(aeg, torch, dist, kernel, n_req=16):
         keys = [gi.kv_key(1, sender, i, l) for i in range(n) for l in range(sh.num_layers)]
         bad, _ = D.verify_chunks(base, offs, keys, sh.chunk_bytes(), seed)
     bad = dist.sum(bad)
+    # the library's copy-engine route (AEG_MIGRATE_CE: gather kernel + CE commands over NVLink, no
+    # SMs on the decode GPU), every pair at once, max-over-ranks device time
+    lib_err = []
+
+    def ce_lib_round():
+        dist.barrier()
+        ms = 0.0
+        if prefill and not lib_err:
+            try:
+                s = new_stream(torch)
+                e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                e0.record(s)
+                ctx.stream_fence(s.cuda_stream)
+                xs = PD.handoff(ctx, sht, src, pairs, rank, dst_by_rank, flags=aeg.MIGRATE_CE)
+                for x in xs.values():
+                    ctx.layer_ready(x, -1, aeg.READY_WAIT_STREAM, s.cuda_stream)
+                e1.record(s)
+                e1.synchronize()
+                for x in xs.values():
+                    ctx.xfer_release(x)
+                ms = e0.elapsed_time(e1)
+            except Exception as e:  # noqa: BLE001  (every rank must still reach the max below)
+                lib_err.append(f"{type(e).__name__}: {e}")
+                ms = -1e9
+        return dist.max(ms)
+    lib_ce_ms = min(ce_lib_round() for _ in range(3))
+    lib_failed = dist.sum(1 if lib_err else 0)
+    lib_ce = ({"error": lib_err[0] if lib_err else "failed on another rank"} if lib_failed or lib_ce_ms <= 0 else
+              {"GBps_aggregate": round(len(pairs) * n * sh.block_bytes() / (lib_ce_ms * 1e6), 1),
+               "GBps_per_pair": round(n * sh.block_bytes() / (lib_ce_ms * 1e6), 1),
+               "what": "aeg_kv_migrate(AEG_MIGRATE_CE): gather kernel into staging, copy-engine commands "
+                       "into the peer pool"})
     # CE-vs-SM: the same chunks paged -> paged, one cudaMemcpyAsync per (block,
     # layer) chunk (copy engines, zero SMs) into the partner's pool mapped here (aeg_peer_region);
     # decode ranks send their chunk offsets.  Max-over-ranks device time of one round, all pairs.
@@ -1256,7 +1295,7 @@ def migrate_leg_dist(aeg, torch, dist, kernel, n_req=16):
     ms = statistics.median(times)
     payload = len(pairs) * n * sh.block_bytes()
     return {"workload": f"configs[2] Llama-2-13B hand-off, {n_req} requests per pair, pairs {pairs}",
-            "nccl_sendrecv_contiguous_baseline": nccl, "per_chunk_ce_route": ce,
+            "nccl_sendrecv_contiguous_baseline": nccl, "per_chunk_ce_route": ce, "library_ce_route": lib_ce,
             "payload_bytes": payload, "ms": round(ms, 3), "GBps_aggregate": round(payload / (ms * 1e6), 1),
             "GBps_per_pair": round(payload / len(pairs) / (ms * 1e6), 1), "peak_per_direction_nominal": NVLINK_NOMINAL,
             "frac_of_nvlink_nominal_per_pair": round(payload / len(pairs) / (ms * 1e6) / NVLINK_NOMINAL, 3),
