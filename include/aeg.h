@@ -162,8 +162,9 @@ typedef struct {
 /* ---- lifecycle -------------------------------------------------------------------------- */
 
 /* Fill *cfg with defaults: 1 GiB slabs (layer-major), 2 GiB stage ring of 64 MiB chunks,
- * 3 x 1 GiB staging slots per direction, 8 host threads, AUTO kernels; region sizes 0.
- * Returns AEG_OK. */
+ * 3 x 1 GiB staging slots per direction, 8 host threads, AUTO kernels; region sizes 0 (a zero
+ * device_kv_bytes is sized at aeg_init from 90% of free VRAM, reading 22; zero host KV / weights
+ * regions are empty).  Returns AEG_OK (INVALID if cfg is NULL). */
 int aeg_config_default(aeg_config* cfg);
 
 /* Create a context on CUDA device `device`: one cudaMalloc for [KV | weights | staging |
