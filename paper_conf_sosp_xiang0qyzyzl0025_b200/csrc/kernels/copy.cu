@@ -231,11 +231,16 @@ __global__ void __launch_bounds__(32) copy_bulk(const CopyArgs a) {
 // once, one per lane (one coalesced block-table load), and lane 0 issues the bulk copies with the
 // pointers broadcast by __shfl_sync; the ring refill is the BULK pipeline (mbarrier complete_tx for
 // loads, bulk_group read-completion before a stage is reloaded).
+// Geometry (tools/small_chunk_probe.cu sweeps, profiles/r02/bulkw_geometry_sweep.txt): 6 warps x
+// 16 KiB of stages in a 96 KiB CTA, one CTA per SM (grid = 148), i.e. 2 stages of 8 KiB pieces per
+// warp and ~96 KiB in flight per SM: 6.3-6.5 TB/s for 8 KiB-320 KiB chunks over 30 GB-spread tables,
+// vs 5.9-6.1 with 192 KiB (4 warps x 48 KiB) or with two CTAs per SM — more bytes or more, smaller
+// bulk copies in flight per SM lose DRAM efficiency on scattered blocks.
 #ifndef AEG_BW_WARPS  // overridable by tools/small_chunk_probe.cu
-#define AEG_BW_WARPS 4
+#define AEG_BW_WARPS 6
 #endif
 #ifndef AEG_BW_SMEM_KIB
-#define AEG_BW_SMEM_KIB 192
+#define AEG_BW_SMEM_KIB 96
 #endif
 constexpr int kBwWarps = AEG_BW_WARPS;
 #ifndef AEG_BW_MAX_STAGES
@@ -342,8 +347,9 @@ cudaError_t launch_t(const CopyArgs& a, int impl, int max_ctas, cudaStream_t s) 
       if (e != cudaSuccess) return e;
       attr_set_w.fetch_or(bit);
     }
-    // whole chunks up to 16 KiB per stage, larger chunks in pieces; at least 2 stages per warp (the
-    // refill of a stage is issued one item after its store, so one stage would never refill)
+    // whole chunks up to 8 KiB per stage (half a warp's share), larger chunks in 8 KiB pieces; at
+    // least 2 stages per warp (the refill of a stage is issued one item after its store, so one
+    // stage would never refill).  One CTA per SM: grid = 148 (the 96 KiB CTA would fit twice).
     const uint32_t cap = std::min<uint32_t>(16u << 10, uint32_t(kBwSmem / kBwWarps / 2) & ~15u);
     const uint32_t piece = a.chunk <= cap ? uint32_t(a.chunk) : cap;
     const uint64_t items = uint64_t(a.nl) * a.n * ((a.chunk + piece - 1) / piece);

@@ -18,13 +18,22 @@ int main() {
   const bool mig = getenv("MIGRATE") != nullptr;  // paged -> paged (H5 local) at large chunks
   std::vector<uint64_t> chunks = {2048ull, 4096ull, 8192ull, 16384ull, 32768ull};
   if (mig) chunks = {32768ull, 262144ull, 327680ull};
+  if (getenv("CHUNKS")) {  // comma-separated override
+    chunks.clear();
+    for (char* p = getenv("CHUNKS"); *p;) {
+      chunks.push_back(strtoull(p, &p, 10));
+      if (*p == ',') ++p;
+    }
+  }
   for (uint64_t chunk : chunks) {
     const int n = int(payload / chunk);
     char *pool, *slot;
-    cudaMalloc(&pool, 2 * payload);  // blocks scattered over twice the payload
+    // blocks scattered over SPREAD x the payload (default 2; SPREAD=30 mimics 30 GB pools)
+    const uint64_t spread = getenv("SPREAD") ? strtoull(getenv("SPREAD"), nullptr, 10) : 2;
+    cudaMalloc(&pool, spread * payload);
     cudaMalloc(&slot, payload);
     std::vector<uint64_t> off(n);
-    for (int i = 0; i < n; ++i) off[i] = uint64_t((uint64_t(i) * 7919) % (2 * n)) * chunk;
+    for (int i = 0; i < n; ++i) off[i] = uint64_t((uint64_t(i) * 7919) % (spread * n)) * chunk;
     std::sort(off.begin(), off.end());
     off.erase(std::unique(off.begin(), off.end()), off.end());
     while (int(off.size()) < n) off.push_back(off.back() + chunk);
@@ -44,7 +53,7 @@ int main() {
       for (int i = n - 1; i > 0; --i) std::swap(off2[i], off2[(uint64_t(i) * 40503u + 7) % (i + 1)]);
       cudaMalloc(&doff2, n * 8);
       cudaMemcpy(doff2, off2.data(), n * 8, cudaMemcpyHostToDevice);
-      cudaMalloc(&pool2, 2 * payload);
+      cudaMalloc(&pool2, spread * payload);
     }
     for (int dir = 0; dir < (mig ? 1 : 2); ++dir) {
       aeg::CopyArgs ca;
@@ -66,26 +75,26 @@ int main() {
       ca.chunk = chunk;
       ca.nl = 1;
       ca.n = n;
-      if (getenv("SWEEP")) {  // BULKW with explicit piece sizes (chunk / 2^k, >= 1 KiB, >= 2 stages)
+      if (getenv("SWEEP")) {  // BULKW with explicit piece sizes (>= 2 stages per warp)
         using namespace aeg;
-        cudaFuncSetAttribute(copy_bulkw<true, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, kBwSmem);
-        cudaFuncSetAttribute(copy_bulkw<false, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, kBwSmem);
-        for (uint64_t piece = chunk; piece >= 1024; piece /= 2) {
-          if (piece * 2 > uint64_t(kBwSmem / kBwWarps)) continue;
+        auto kern = mig ? copy_bulkw<true, true> : dir == 0 ? copy_bulkw<true, false> : copy_bulkw<false, true>;
+        cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, kBwSmem);
+        std::vector<uint64_t> pieces = {chunk, 16384, 12288, 10240, 8192, 6144, 5120, 4096, 2048};
+        std::sort(pieces.begin(), pieces.end());
+        pieces.erase(std::unique(pieces.begin(), pieces.end()), pieces.end());
+        for (uint64_t piece : pieces) {
+          if (piece > chunk || piece * 2 > uint64_t(kBwSmem / kBwWarps)) continue;
           const uint64_t items = uint64_t(n) * ((chunk + piece - 1) / piece);
-          const int smp = 2 * 1024 * 1024 / 1;  // unused
-          (void)smp;
           int occ = 0;
-          cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, copy_bulkw<true, false>, kBwWarps * 32, kBwSmem);
-          uint64_t grid = uint64_t(148) * std::max(1, occ);
+          cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kern, kBwWarps * 32, kBwSmem);
+          // CTAS_PER_SM caps the grid below the occupancy limit (in-flight bulk copies per SM)
+          const int cps = getenv("CTAS_PER_SM") ? atoi(getenv("CTAS_PER_SM")) : occ;
+          uint64_t grid = uint64_t(148) * std::max(1, std::min(occ, cps));
           if (grid > (items + kBwWarps - 1) / kBwWarps) grid = (items + kBwWarps - 1) / kBwWarps;
           std::vector<float> ts;
           for (int r = 0; r < 12; ++r) {
             cudaEventRecord(a, s);
-            if (dir == 0)
-              copy_bulkw<true, false><<<unsigned(grid), kBwWarps * 32, kBwSmem, s>>>(ca, uint32_t(piece));
-            else
-              copy_bulkw<false, true><<<unsigned(grid), kBwWarps * 32, kBwSmem, s>>>(ca, uint32_t(piece));
+            kern<<<unsigned(grid), kBwWarps * 32, kBwSmem, s>>>(ca, uint32_t(piece));
             cudaEventRecord(b, s);
             cudaEventSynchronize(b);
             float ms;
@@ -95,7 +104,8 @@ int main() {
           std::sort(ts.begin(), ts.end());
           const double med = ts[ts.size() / 2];
           printf("chunk=%6llu %s BULKW warps=%d smem=%dK ctas/SM=%d piece=%6llu median %8.1f us  %7.0f GB/s\n",
-                 (unsigned long long)chunk, mig ? "migrate" : dir ? "scatter" : "gather ", kBwWarps, kBwSmem >> 10, occ,
+                 (unsigned long long)chunk, mig ? "migrate" : dir ? "scatter" : "gather ", kBwWarps, kBwSmem >> 10,
+                 int(grid / 148),
                  (unsigned long long)piece, med * 1e3, 2.0 * payload / (med * 1e6));
         }
         continue;
