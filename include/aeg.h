@@ -85,10 +85,11 @@ enum {
                                    the node-shared "Unified CPU KV Cache" (Fig. 5) */
 };
 /* kernel selection for gather/scatter/migrate.  AEG_KERNEL_AUTO picks the measured best by chunk
- * size Cl (profiles/r02/small_chunk_*.txt): gather/scatter WARP if Cl <= 2 KiB, BULKW
- * (bulk copies issued by several warps per CTA) if Cl <= 16 KiB, BULK otherwise; migrate (paged ->
- * paged) WARP if Cl <= 4 KiB, else BULKW within this process's pools on this GPU and LSU (16-byte
- * stores) into another process's or another GPU's pool. */
+ * size Cl (profiles/r02/): gather/scatter WARP if Cl <= 2 KiB, otherwise BULKW (bulk
+ * copies issued by 6 warps per CTA, one CTA per SM); migrate (paged -> paged) WARP if Cl <= 4 KiB,
+ * else BULKW within this process's pools on this GPU and LSU (16-byte stores) into another
+ * process's or another GPU's pool.  LSU / BULK (one issuing thread per CTA) / WARP / BULKW can be
+ * forced for every launch. */
 enum { AEG_KERNEL_AUTO = 0, AEG_KERNEL_LSU = 1, AEG_KERNEL_BULK = 2, AEG_KERNEL_WARP = 3, AEG_KERNEL_BULKW = 4 };
 
 /* ---- structs ---------------------------------------------------------------------------- */

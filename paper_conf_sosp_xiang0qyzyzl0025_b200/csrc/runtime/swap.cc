@@ -246,25 +246,24 @@ static void host_dmas(const SlabPool& hp, char* hbase, const Shape& sh, const st
   }
 }
 
-// AUTO = BULK (cp.async.bulk through shared memory): measured 5.93 TB/s in-step for the C2 gather vs
-// 5.56 TB/s for LSU with 1 GiB slots (profiles/r01).  Stores into another GPU's pool use LSU under AUTO
-// (plain st.global to peer addresses) unless BULK is requested explicitly.
+// Under AUTO every gather/scatter above 2 KiB chunks uses BULKW (cp.async.bulk issued by 6 warps per
+// CTA).  Stores into another GPU's pool use LSU under AUTO (plain st.global to peer addresses).
 #define ipc_events(flags) (((flags) & AEG_IPC_EVENTS) || (cfg.flags & AEG_CFG_SHARED_HOST))
 
-// AUTO by chunk size, from tools/small_chunk_probe.cu (profiles/r02/small_chunk_probe.txt, 1 GiB
-// gather / scatter launches, median TB/s) and tools/threshold_probe.cu (profiles/r01):
-//   2 KiB: WARP 5.96 / 6.01, BULKW 5.63 / 5.62, LSU 1.8, BULK 0.8
-//   4 KiB: BULKW 5.86 / 5.90, WARP 5.57 / 5.62, LSU 3.4-3.5
-//   8 KiB: BULKW 5.98 / 5.91, WARP 5.70 / 5.74, LSU 5.46 / 5.50, BULK 2.99 / 2.93
-//   16 KiB: BULKW 6.04 / 6.00, LSU 6.03 / 5.91, BULK 5.13 / 5.15
-//   32 KiB: BULK 5.98 / 6.14, BULKW 6.03 / 6.00, LSU 5.76 / 5.80;  64-512 KiB: BULK 6.1-6.5, LSU 5.9
+// AUTO by chunk size, from tools/small_chunk_probe.cu (profiles/r02/small_chunk_probe_final_bulkw.txt, 1 GiB
+// gather / scatter launches over 30 GB-spread tables, median TB/s) and the bench's own C2 step:
+//   2 KiB: WARP 5.97 / 6.08, BULKW 5.47 / 5.51, LSU 1.8, BULK 0.8
+//   4 KiB: BULKW 5.98 / 5.93, WARP 5.56 / 5.63, LSU 3.4-3.5
+//   8 KiB: BULKW 6.26 / 6.36, WARP 5.74, LSU 5.48, BULK 2.99
+//   16-32 KiB: BULKW 6.33-6.47, LSU 5.8-6.1, BULK 5.1-6.1;  256 KiB: BULKW 6.47 / 6.44, BULK 6.1
+//   C2 step in-step (256 KiB chunks, 1 GiB launches next to PCIe DMA): BULKW 5.91 / 5.81 TB/s
+//   gather / scatter vs BULK 5.73 / 5.53 (profiles/r02/bench_bulkw_vs_bulk.txt)
 static int impl_of(const aeg_config& cfg, uint64_t chunk) {
   if (cfg.kernel == AEG_KERNEL_LSU) return IMPL_LSU;
   if (cfg.kernel == AEG_KERNEL_BULK) return IMPL_BULK;
   if (cfg.kernel == AEG_KERNEL_WARP) return IMPL_WARP;
   if (cfg.kernel == AEG_KERNEL_BULKW) return IMPL_BULKW;
-  if (chunk <= (2u << 10)) return IMPL_WARP;
-  return chunk <= (16u << 10) ? IMPL_BULKW : IMPL_BULK;
+  return chunk <= (2u << 10) ? IMPL_WARP : IMPL_BULKW;
 }
 
 // Optional host-side phase timer of swap_out (AEG_HOST_PROFILE=1: totals printed at exit): where
