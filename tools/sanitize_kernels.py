@@ -20,6 +20,7 @@ for shape in [(1, 1, 8, 2, 1), (3, 1, 8, 2, 1), (1, 2, 64, 2, 16)]:
         E.test_small_shapes_round_trip(shape, k)
         n += 1
 for k in (aeg.KERNEL_AUTO, aeg.KERNEL_BULKW):
-    M.test_local_migrate(k)
-    n += 1
+    for ce in (False, True):          # fused kernel / copy-engine route
+        M.test_local_migrate(k, ce)
+        n += 1
 print(f"{n} oracle-checked cases passed")
