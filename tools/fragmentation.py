@@ -67,6 +67,10 @@ def run(ev, pool_bytes: int, slab_bytes: int):
     live, oom = {}, 0
     samples = []
     peak = (0, 0, None)
+    names = [n for n, _, _, _ in SHAPES]
+    block = {n: L * 2 * H * D * 2 * 16 for n, L, H, D in SHAPES}
+    shape_peak = {n: 0 for n in names}        # per-shape peak allocated (assigned slab) bytes
+    shape_frag = {n: [] for n in names}       # per-shape unused / peak allocated, at every event
     for e in ev:
         if e[1] == "a":
             _, _, m, r, nb = e
@@ -81,6 +85,16 @@ def run(ev, pool_bytes: int, slab_bytes: int):
                 ctx.kv_free(aeg.POOL_HOST, live.pop(r))
         s = ctx.stats(aeg.POOL_HOST)
         samples.append((s.assigned_bytes, s.used_bytes, s.peak_assigned_bytes))
+        cur = {}
+        for i in range(s.n_shapes):
+            p = s.per_shape[i]
+            nm = [n for n, L_, H, D in SHAPES if L_ == p.shape.num_layers and H == p.shape.num_kv_heads][0]
+            cur[nm] = (p.slabs * slab_bytes, p.owned_blocks * block[nm])
+        for nm in names:
+            asg, used = cur.get(nm, (0, 0))
+            shape_peak[nm] = max(shape_peak[nm], asg)
+            if shape_peak[nm]:
+                shape_frag[nm].append((asg - used) / shape_peak[nm])
         if s.assigned_bytes > peak[0]:
             per = {}
             for i in range(s.n_shapes):
@@ -96,6 +110,8 @@ def run(ev, pool_bytes: int, slab_bytes: int):
     frag = (a[:, 0] - a[:, 1]) / a[:, 2]       # Fig. 16: unused / peak allocated, at every event
     occ = a[:, 1] / pool_bytes
     return {"slab_GiB": slab_bytes / GIB, "events": len(ev), "oom_allocs": oom,
+            "per_shape_frag_unused_over_peak_allocated_mean": {
+                n: round(float(np.mean(v[len(v) // 10:])), 4) for n, v in shape_frag.items() if v},
             "occupancy_used_over_pool_mean": round(float(occ.mean()), 4),
             "occupancy_used_over_pool_max": round(float(occ.max()), 4),
             "frag_unused_over_peak_allocated_mean": round(float(frag.mean()), 4),
