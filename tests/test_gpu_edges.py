@@ -167,3 +167,38 @@ def test_default_device_kv_takes_90pct_of_free_vram():
         ctx.kv_free(aeg.POOL_DEVICE, b)
     finally:
         ctx.shutdown()
+
+
+def test_readme_example_round_trip():
+    """The README's minimal use of the binding (default 90 %-of-free-VRAM device pool, Qwen-7B shape,
+    128 blocks out and back with per-layer stream waits) moves every chunk back intact."""
+    require_gpu()
+    import torch
+    from aeg_inputs import dev as Dv
+    ctx = aeg.Context(0, aeg.default_config(host_kv_bytes=2 << 30))
+    try:
+        qwen7b = (32, 32, 128, 2, 16)
+        sh = KVShape(*qwen7b)
+        dev = ctx.kv_alloc(aeg.POOL_DEVICE, qwen7b, 128)
+        host = ctx.kv_alloc(aeg.POOL_HOST, qwen7b, 128)
+        base, _ = ctx.pool_region(aeg.POOL_DEVICE)
+
+        def offs(blocks):
+            o0, ls = ctx.block_offsets(aeg.POOL_DEVICE, qwen7b, blocks)
+            return [int(o) + l * int(ls) for o in o0 for l in range(sh.L)]
+        keys = [gi.kv_key(9, 0, i, l) for i in range(128) for l in range(sh.L)]
+        seed = gi.kv_seed(1)
+        Dv.fill_chunks(base, offs(dev), keys, sh.chunk_bytes(), seed)
+        x = ctx.kv_swap_out(qwen7b, dev, host, flags=aeg.FREE_SRC)
+        back = ctx.kv_alloc(aeg.POOL_DEVICE, qwen7b, 128)
+        y = ctx.kv_swap_in(qwen7b, host, back, flags=aeg.FREE_SRC)
+        decode_stream = torch.cuda.Stream()
+        for l in range(32):
+            ctx.layer_ready(y, l, aeg.READY_WAIT_STREAM, decode_stream.cuda_stream)
+        decode_stream.synchronize()
+        bad, first = Dv.verify_chunks(base, offs(back), keys, sh.chunk_bytes(), seed)
+        assert bad == 0, first
+        ctx.xfer_release(x)
+        ctx.xfer_release(y)
+    finally:
+        ctx.shutdown()
