@@ -74,6 +74,7 @@ def parse():
     p.add_argument("--slots", type=int, default=0)
     p.add_argument("--dma-piece-mib", type=int, default=0, help="swap-out D2H piece (0 = library default)")
     p.add_argument("--profile", action="store_true", help="short run for ncu (no side legs)")
+    p.add_argument("--two-device-probe", action="store_true", help=argparse.SUPPRESS)
     return p.parse_args()
 
 
@@ -2004,6 +2005,9 @@ def run_ours(args):
             if rank == 0 and dist.local == 0:   # the cross-device branch of aeg_import_peer, one process
                 mig["two_device_same_process"] = leg("migrate_two_device",
                                                      lambda: migrate_leg_two_device(aeg, torch, kernel))
+                # bulk copies (cp.async.bulk) storing into another GPU's memory are not relied on by
+                # AUTO; measure them in a throw-away process so a fault cannot touch this one
+                mig["two_device_bulkw_stores_probe"] = leg("two_device_bulkw", two_device_bulkw_probe)
             dist.barrier()
         else:
             mig = leg("migrate", lambda: migrate_leg(aeg, torch, kernel, args.migrate_requests))
@@ -2091,8 +2095,28 @@ def run_ours(args):
     return 0
 
 
+def two_device_bulkw_probe(timeout_s=300):
+    """Run migrate_leg_two_device with the BULKW kernel forced (bulk stores into the peer GPU) in a
+    separate process; returns its JSON or what went wrong."""
+    env = {k: v for k, v in os.environ.items() if k not in ("RANK", "LOCAL_RANK", "WORLD_SIZE")}
+    try:
+        r = subprocess.run([sys.executable, os.path.abspath(__file__), "--two-device-probe"], capture_output=True,
+                           text=True, timeout=timeout_s, env=env)
+    except subprocess.TimeoutExpired:
+        return {"error": f"timed out after {timeout_s} s"}
+    for line in reversed(r.stdout.splitlines()):
+        if line.startswith("{"):
+            return json.loads(line)
+    return {"error": f"rc {r.returncode}", "stderr_tail": r.stderr[-400:]}
+
+
 def main():
     args = parse()
+    if args.two_device_probe:
+        import torch
+        import paper_conf_sosp_xiang0qyzyzl0025_b200 as aeg
+        print(json.dumps(migrate_leg_two_device(aeg, torch, aeg.KERNEL_BULKW)), flush=True)
+        return 0
     if args.impl == "reference":
         return run_reference(args)
     return run_ours(args)
