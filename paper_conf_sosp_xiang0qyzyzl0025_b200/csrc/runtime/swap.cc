@@ -604,6 +604,8 @@ uint64_t Ctx::migrate(const Shape& sh, const aeg_block* src, int32_t peer, const
     dg = &P->geom;
     dbase = P->dev_kv;
   }
+  AEG_REQUIRE(!(flags & AEG_MIGRATE_CE) || sh.chunk() <= ring_out.slot_bytes, AEG_ERR_INVALID,
+              "copy-engine route: chunk larger than a staging slot");
   Xfer* x = new_xfer(X_MIGRATE, sh.L, ipc_events(flags) || (peer >= 0 && !P->same_process));
   std::vector<uint64_t> rdeps, wdeps;
   if (!(flags & AEG_NO_DEPS)) {
@@ -634,7 +636,6 @@ uint64_t Ctx::migrate(const Shape& sh, const aeg_block* src, int32_t peer, const
       for (int32_t i = 0; i < n; ++i) t[i] = dp.off0(src[i], sh);
       fetch_table(dtab, htab, uint64_t(n) * 8, s_gather);
     }
-    AEG_REQUIRE(sh.chunk() <= ring_out.slot_bytes, AEG_ERR_INVALID, "chunk larger than a staging slot");
     const auto segs = plan(sh.L, n, sh.chunk(), ring_out.slot_bytes);
     const auto runs = runs_of(dst, n);
     const uint64_t sstride = dp.lstride(sh);

@@ -29,7 +29,8 @@ def test_empty_transfers_are_ready():
     ctx, _, _ = make()
     try:
         sh = (2, 1, 64, 2, 16)
-        for x in (ctx.kv_swap_out(sh, [], []), ctx.kv_swap_in(sh, [], []), ctx.kv_migrate(sh, [], -1, [])):
+        for x in (ctx.kv_swap_out(sh, [], []), ctx.kv_swap_in(sh, [], []), ctx.kv_migrate(sh, [], -1, []),
+                  ctx.kv_migrate(sh, [], -1, [], flags=aeg.MIGRATE_CE)):
             ctx.layer_ready(x, -1, aeg.READY_BLOCK)
             assert all(ctx.layer_ready(x, l, aeg.READY_QUERY) for l in range(2))
             ctx.xfer_release(x)
@@ -60,6 +61,25 @@ def test_small_shapes_round_trip(shape, kernel):
         ctx.layer_ready(y, -1, aeg.READY_BLOCK)
         dimg = OK.swap_in(himg, host.geom, dimg, dev.geom, sh, ho, no)
         assert first_diff(dev.read(), dimg) is None
+    finally:
+        ctx.shutdown()
+
+
+def test_copy_engine_route_rejects_a_chunk_larger_than_a_slot():
+    """AEG_MIGRATE_CE stages through the out ring: a chunk above staging_slot_bytes is INVALID and
+    changes nothing (the fused kernel route has no such limit)."""
+    require_gpu()
+    ctx, dev, _ = make(slab=4 * MIB, dev_slabs=4)
+    try:
+        big = KVShape(1, 32, 128, 2, 128)        # chunk = 2 MiB > the 1 MiB slot
+        sc, so = dev.alloc(big, 1)
+        dc, do = dev.alloc(big, 1)
+        with pytest.raises(aeg.AegError) as e:
+            ctx.kv_migrate(big.as_tuple(), sc, -1, dc, flags=aeg.MIGRATE_CE)
+        assert e.value.code == aeg.ERR_INVALID
+        x = ctx.kv_migrate(big.as_tuple(), sc, -1, dc)   # the kernel route copies it
+        ctx.layer_ready(x, -1, aeg.READY_BLOCK)
+        ctx.xfer_release(x)
     finally:
         ctx.shutdown()
 
