@@ -164,3 +164,94 @@ def test_c3_full_size_handoff():
     finally:
         a.shutdown()
         b.shutdown()
+
+
+def test_c4_full_size_three_model_switch():
+    """configs[3] at full size: Qwen-1.8B / Llama-7B / Yi-9B weights (3.7 / 13.5 / 17.7 GB, generated
+    pageable Model Caches) with 1 GiB of KV each, switched A -> B -> C -> A in the production order
+    (B's KV in, B's weights staged through the Stage Buffer, a per-layer consumer wait, A's KV out
+    fenced after it).  After every switch: every KV chunk of every
+    model — on the device or in the host pool — equals the generator's content at the library's
+    block table (O5/O6: a swap is the identity under relabelling), and the running model's weights
+    equal oracle O8 (TP = 1: the tensors at the bump offsets) on 14 sampled tensors."""
+    require_gpu()
+    import torch
+    GIB = 1 << 30
+    names = ["qwen-1.8b", "llama-7b", "yi-9b"]
+    seed = gi.kv_seed(4)
+    models = []
+    wmax = 0
+    for m, nm in enumerate(names):
+        ts = gi.model_tensors(nm)
+        sizes = [t["rows"] * t["cols"] * 2 for t in ts]
+        offs = np.cumsum([0] + [-(-s // 256) * 256 for s in sizes])
+        buf = np.empty(int(offs[-1]), dtype=np.uint8)
+        for k, (o, s) in enumerate(zip(offs, sizes)):
+            D.host_fill(buf[o:o + s], gi.w_seed(6), gi.weight_key(10 + m, k), threads=16)
+        descs = [dict(host_src=buf.ctypes.data + int(o), rows=t["rows"], cols=t["cols"], elem_bytes=2,
+                      layer=t["layer"], split=t["split"], groups=t["groups"]) for t, o in zip(ts, offs)]
+        sht = gi.KV_SHAPES[nm]
+        L, H, Dh, s_, B = sht
+        n = GIB // (L * 2 * H * Dh * s_ * B)
+        models.append(dict(name=nm, ts=ts, sizes=sizes, offs=offs, buf=buf, descs=descs, sht=sht, n=n,
+                           keys=[gi.kv_key(20 + m, 0, i, l) for i in range(n) for l in range(L)]))
+        wmax = max(wmax, int(offs[-1]))
+    ctx = aeg.Context(0, aeg.default_config(device_kv_bytes=8 * GIB, host_kv_bytes=8 * GIB,
+                                            device_weight_bytes=wmax + (64 << 20), host_threads=12))
+    try:
+        dbase, _ = ctx.pool_region(aeg.POOL_DEVICE)
+        hbase, _ = ctx.pool_region(aeg.POOL_HOST)
+        wbase, _, _ = ctx.weights_region()
+
+        def chunk_offs(pool, M, blocks):
+            o0, ls = ctx.block_offsets(pool, M["sht"], blocks)
+            return [int(o) + l * int(ls) for o in o0 for l in range(M["sht"][0])]
+
+        def check_kv():
+            for M in models:
+                pool, base = (aeg.POOL_DEVICE, dbase) if M["where"] == "dev" else (aeg.POOL_HOST, hbase)
+                bad, first = D.verify_chunks(base, chunk_offs(pool, M, M["blocks"]), M["keys"],
+                                             aeg.KVShape.of(M["sht"]).chunk_bytes(), seed)
+                assert bad == 0, (M["name"], M["where"], first)
+
+        for M in models:   # every model's decode KV starts in the host pool
+            M["blocks"] = ctx.kv_alloc(aeg.POOL_HOST, M["sht"], M["n"])
+            M["where"] = "host"
+            D.fill_chunks(hbase, chunk_offs(aeg.POOL_HOST, M, M["blocks"]), M["keys"],
+                          aeg.KVShape.of(M["sht"]).chunk_bytes(), seed)
+        cons = torch.cuda.Stream()
+        rng = np.random.default_rng(4)
+        cur = None
+        for b in [0, 1, 2, 0]:
+            B_, A_ = models[b], (models[cur] if cur is not None else None)
+            db = ctx.kv_alloc(aeg.POOL_DEVICE, B_["sht"], B_["n"])
+            ctx.stream_fence(cons.cuda_stream)
+            xi = ctx.kv_swap_in(B_["sht"], B_["blocks"], db, flags=aeg.FREE_SRC)
+            ctx.weights_reset(0)
+            woffs, xw = ctx.weights_stage(B_["descs"])
+            for l in range(B_["sht"][0]):
+                ctx.layer_ready(xi, l, aeg.READY_WAIT_STREAM, cons.cuda_stream)
+            ctx.layer_ready(xw, -1, aeg.READY_WAIT_STREAM, cons.cuda_stream)
+            xo = None
+            if A_ is not None:
+                ctx.stream_fence(cons.cuda_stream)
+                hb = ctx.kv_alloc(aeg.POOL_HOST, A_["sht"], A_["n"])
+                xo = ctx.kv_swap_out(A_["sht"], A_["blocks"], hb, flags=aeg.FREE_SRC)
+            for x in (xi, xw, xo):
+                if x is not None:
+                    ctx.layer_ready(x, -1, aeg.READY_BLOCK)
+                    ctx.xfer_release(x)
+            B_.update(blocks=db, where="dev")
+            if A_ is not None:
+                A_.update(blocks=hb, where="host")
+            check_kv()
+            exp_offs, _ = W.bump_offsets(B_["sizes"], 0)
+            assert [int(o) for o in woffs] == exp_offs
+            nt = len(B_["ts"])
+            for k in sorted(set([0, nt - 1] + rng.choice(nt, 12, replace=False).tolist())):
+                nbytes = min(B_["sizes"][k], 1 << 24)
+                got = D.read(wbase + exp_offs[k], nbytes)
+                assert np.array_equal(got, B_["buf"][B_["offs"][k]:B_["offs"][k] + nbytes]), (B_["name"], k)
+            cur = b
+    finally:
+        ctx.shutdown()
