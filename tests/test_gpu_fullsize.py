@@ -194,7 +194,7 @@ def test_c4_full_size_three_model_switch():
         L, H, Dh, s_, B = sht
         n = GIB // (L * 2 * H * Dh * s_ * B)
         models.append(dict(name=nm, ts=ts, sizes=sizes, offs=offs, buf=buf, descs=descs, sht=sht, n=n,
-                           keys=[gi.kv_key(20 + m, 0, i, l) for i in range(n) for l in range(L)]))
+                           keys=[gi.kv_key(11 + m, 0, i, l) for i in range(n) for l in range(L)]))
         wmax = max(wmax, int(offs[-1]))
     ctx = aeg.Context(0, aeg.default_config(device_kv_bytes=8 * GIB, host_kv_bytes=8 * GIB,
                                             device_weight_bytes=wmax + (64 << 20), host_threads=12))
