@@ -52,7 +52,7 @@ def descs_for(buf_tens, descs):
                  split=d["split"], groups=d["groups"]) for t, d in zip(buf_tens, descs)]
 
 
-@pytest.mark.parametrize("tp", [1, 2, 4])
+@pytest.mark.parametrize("tp", [1, 2, 4, 8])
 @pytest.mark.parametrize("direct", [False, True])
 @pytest.mark.parametrize("arch", ["llama", "qwen1"])      # qwen1: fused QKV, COL split per group of 3
 def test_stage_matches_oracle(tp, direct, arch):
