@@ -59,7 +59,7 @@ int main() {
     ca.nl = 1;
     ca.n = n;
     const double alg = 2.0 * n * chunk;
-    for (int impl : {aeg::IMPL_LSU, aeg::IMPL_BULK, aeg::IMPL_WARP}) {
+    for (int impl : {aeg::IMPL_LSU, aeg::IMPL_BULK, aeg::IMPL_WARP, aeg::IMPL_BULKW}) {
       for (char mode : {'A', 'C'}) {
         double tot = 0, span = 0;
         const int R = 20;
@@ -88,7 +88,7 @@ int main() {
           }
         }
         printf("chunk=%6llu n=%5d %s %c  event %.1f us (%.0f GB/s)   stamp-to-stamp %.1f us (%.0f GB/s)\n",
-               (unsigned long long)chunk, n, impl == aeg::IMPL_LSU ? "LSU " : impl == aeg::IMPL_BULK ? "BULK" : "WARP",
+               (unsigned long long)chunk, n, impl == aeg::IMPL_LSU ? "LSU " : impl == aeg::IMPL_BULK ? "BULK" : impl == aeg::IMPL_WARP ? "WARP" : "BLKW",
                mode, 1e3 * tot / R, alg / (tot / R) / 1e6, 1e3 * span / R, alg / (span / R) / 1e6);
       }
     }
