@@ -1780,6 +1780,68 @@ def overlap_leg(aeg, torch, kernel, work_us=500, reps=5):
     return out
 
 
+def per_request_sync_leg(aeg, torch, kernel, h2d_GBps=None, n_req=32):
+    """Fig. 15 (right) on B200: the per-request KV cache transfer overhead.  n_req
+    Qwen-7B requests with ShareGPT-like lengths (lognormal prompt + output, seeded) sit in the host
+    pool; the scheduler issues one swap-in per request back to back (per-request transfers and
+    readiness) and the decode side waits per request.  Per request: device time
+    from the first issue to its last layer ready; its ideal is the cumulative bytes over the plain
+    H2D memcpy rate of this box; overhead = ready - ideal.  Also the host enqueue time per call."""
+    import aeg_inputs as gi
+    sh = QWEN7B
+    bb = aeg.KVShape.of(sh).block_bytes()
+    g = gi.rng(31)
+    lens = [int(g.lognormal(np.log(600), 0.8)) + int(g.lognormal(np.log(300), 0.8)) for _ in range(n_req)]
+    nblk = [-(-max(1, t) // 16) for t in lens]
+    ctx = aeg.Context(0, aeg.default_config(device_kv_bytes=(sum(nblk) * bb // GIB + 4) * GIB,
+                                            host_kv_bytes=(sum(nblk) * bb // GIB + 4) * GIB, kernel=kernel))
+    try:
+        host = [ctx.kv_alloc(aeg.POOL_HOST, sh, n) for n in nblk]
+        cons = new_stream(torch)
+        rows = []
+        for rep in range(3):
+            dev = [ctx.kv_alloc(aeg.POOL_DEVICE, sh, n) for n in nblk]
+            torch.cuda.synchronize()
+            e0 = torch.cuda.Event(enable_timing=True)
+            e0.record(cons)
+            ctx.stream_fence(cons.cuda_stream)
+            xs, evs, enq = [], [], []
+            for h, d in zip(host, dev):
+                t0 = time.perf_counter()
+                xs.append(ctx.kv_swap_in(sh, h, d))
+                enq.append((time.perf_counter() - t0) * 1e6)
+                # the decode side waits for this request right away (an event recorded later would
+                # time the host's enqueue, not the request): ready = its last layer has landed
+                ctx.layer_ready(xs[-1], -1, aeg.READY_WAIT_STREAM, cons.cuda_stream)
+                e = torch.cuda.Event(enable_timing=True)
+                e.record(cons)
+                evs.append(e)
+            evs[-1].synchronize()
+            ready = [e0.elapsed_time(e) for e in evs]
+            for x in xs:
+                ctx.xfer_release(x)
+            for d in dev:
+                ctx.kv_free(aeg.POOL_DEVICE, d)
+            if rep:
+                rows.append((ready, enq))
+    finally:
+        ctx.shutdown()
+    ready = [statistics.median(r[0][i] for r in rows) for i in range(n_req)]
+    enq = sorted(e for r in rows for e in r[1])
+    cum = np.cumsum([n * bb for n in nblk])
+    out = {"workload": f"{n_req} Qwen-7B requests, ShareGPT-like lengths (mean {int(np.mean(lens))} tokens, "
+                       f"{sum(nblk)} blocks, {cum[-1] / GIB:.2f} GiB), one swap-in per request, back to back",
+           "ready_ms_p50": round(float(np.median(ready)), 2), "ready_ms_max": round(max(ready), 2),
+           "per_request_transfer_ms_p50": round(float(np.median(np.diff([0.0] + ready))), 3),
+           "enqueue_us_p50": round(enq[len(enq) // 2], 1), "enqueue_us_p90": round(enq[int(0.9 * (len(enq) - 1))], 1),
+           "GBps": round(cum[-1] / (ready[-1] * 1e6), 1)}
+    if h2d_GBps:
+        over = [r - c / (h2d_GBps * 1e6) for r, c in zip(ready, cum)]
+        out.update({"overhead_vs_memcpy_ms_p50": round(float(np.median(over)), 3),
+                    "overhead_vs_memcpy_ms_max": round(max(over), 3), "h2d_memcpy_GBps": h2d_GBps})
+    return out
+
+
 class OracleSample:
     """The oracle as it stands (NumPy, one host core for its copies) on a bounded, resident sample
     of the C2 workload: swap-out + swap-in of `blocks` Qwen-7B blocks between byte-image pools
@@ -2024,6 +2086,8 @@ def run_ours(args):
                   "model_cache_gen_s": round(gen_s, 1)}
             del caches
         ovl = None if args.no_switch or world > 1 else leg("overlap", lambda: overlap_leg(aeg, torch, kernel))
+        prs = None if world > 1 else leg("per_request_sync", lambda: per_request_sync_leg(
+            aeg, torch, kernel, h2d_GBps=pc.get("h2d")))
         if args.no_c5:
             c5 = None
         elif world in (1, 8):
@@ -2038,7 +2102,8 @@ def run_ours(args):
         alloc = leg("allocator", lambda: allocator_leg(aeg)) if rank == 0 else None
         cpu = None if args.no_cpu or rank != 0 else leg("cpu_baseline", cpu_baseline)
         out.update({"e2e": e2e, "verify": ver, "one_direction": one_dir, "pcie_memcpy_GBps": {k: round(v, 1) for k, v in pc.items()},
-                    "switch": sw, "migrate": mig, "per_layer_overlap": ovl, "c5": c5, "allocator": alloc,
+                    "switch": sw, "migrate": mig, "per_layer_overlap": ovl, "per_request_sync": prs, "c5": c5,
+                    "allocator": alloc,
                     "per_chunk_memcpy_baseline": base, "small_chunk": small, "small_chunk_tp4": small_tp4, "c1": c1, "back_to_back": back2back,
                     "host_route": route,
                     "host": host_facts(),
