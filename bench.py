@@ -1838,7 +1838,7 @@ def per_request_sync_leg(aeg, torch, kernel, h2d_GBps=None, n_req=32):
     if h2d_GBps:
         over = [r - c / (h2d_GBps * 1e6) for r, c in zip(ready, cum)]
         out.update({"overhead_vs_memcpy_ms_p50": round(float(np.median(over)), 3),
-                    "overhead_vs_memcpy_ms_max": round(max(over), 3), "h2d_memcpy_GBps": h2d_GBps})
+                    "overhead_vs_memcpy_ms_max": round(max(over), 3), "h2d_memcpy_GBps": round(h2d_GBps, 1)})
     return out
 
 
