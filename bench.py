@@ -1730,7 +1730,7 @@ def allocator_leg(aeg, reps=20):
             "one_block_call_us_p50": med(one), "includes": "Python ctypes call overhead"}
 
 
-def overlap_leg(aeg, torch, kernel, work_us=500, reps=5):
+def overlap_leg(aeg, torch, kernel, work_us=500, reps=5, pack_mib=0):
     """North star: "decoding of layer i overlaps the transfer of layer i+1".  A 1 GiB Llama-7B KV
     batch (32 layers) is swapped in while a synthetic decode step does `work_us` of work per layer
     (a spin kernel ~ one layer of a 7B decode step).  per_layer: layer l's work waits only on layer
@@ -1742,7 +1742,8 @@ def overlap_leg(aeg, torch, kernel, work_us=500, reps=5):
     sh = gi.KV_SHAPES["llama-7b"]
     bb = sh[0] * 2 * sh[1] * sh[2] * sh[3] * sh[4]
     n = GIB // bb
-    ctx = aeg.Context(0, aeg.default_config(device_kv_bytes=4 * GIB, host_kv_bytes=4 * GIB, kernel=kernel))
+    ctx = aeg.Context(0, aeg.default_config(device_kv_bytes=4 * GIB, host_kv_bytes=4 * GIB, kernel=kernel,
+                                            pack_layer_mib=pack_mib))
     # clock64 cycles per microsecond at the current SM clock
     cyc_per_us = torch.cuda.get_device_properties(0).clock_rate / 1e3 if hasattr(
         torch.cuda.get_device_properties(0), "clock_rate") else 1965.0
@@ -1780,7 +1781,7 @@ def overlap_leg(aeg, torch, kernel, work_us=500, reps=5):
     return out
 
 
-def per_request_sync_leg(aeg, torch, kernel, h2d_GBps=None, n_req=32):
+def per_request_sync_leg(aeg, torch, kernel, h2d_GBps=None, n_req=32, pack_mib=0):
     """Fig. 15 (right) on B200: the per-request KV cache transfer overhead.  n_req
     Qwen-7B requests with ShareGPT-like lengths (lognormal prompt + output, seeded) sit in the host
     pool; the scheduler issues one swap-in per request back to back (per-request transfers and
@@ -1794,7 +1795,8 @@ def per_request_sync_leg(aeg, torch, kernel, h2d_GBps=None, n_req=32):
     lens = [int(g.lognormal(np.log(600), 0.8)) + int(g.lognormal(np.log(300), 0.8)) for _ in range(n_req)]
     nblk = [-(-max(1, t) // 16) for t in lens]
     ctx = aeg.Context(0, aeg.default_config(device_kv_bytes=(sum(nblk) * bb // GIB + 4) * GIB,
-                                            host_kv_bytes=(sum(nblk) * bb // GIB + 4) * GIB, kernel=kernel))
+                                            host_kv_bytes=(sum(nblk) * bb // GIB + 4) * GIB, kernel=kernel,
+                                            pack_layer_mib=pack_mib))
     try:
         host = [ctx.kv_alloc(aeg.POOL_HOST, sh, n) for n in nblk]
         cons = new_stream(torch)

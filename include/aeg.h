@@ -131,7 +131,10 @@ typedef struct {
                                    boundaries; very small pieces on big transfers can exceed the
                                    ~1,000 pending copies a stream holds, and the data call then
                                    blocks until the copy engine drains (correct, not async)      */
-  uint32_t reserved[5];
+  uint32_t pack_layer_mib;      /* KV swaps: layers smaller than this share one staging segment
+                                   (one kernel launch, fewer copy commands, readiness per
+                                   segment); 0 = the default                      */
+  uint32_t reserved[4];
 } aeg_config;
 
 /* One checkpoint tensor in the (pageable or registered) host Model Cache, row-major

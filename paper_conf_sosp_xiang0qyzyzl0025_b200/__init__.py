@@ -62,7 +62,7 @@ class Config(C.Structure):
                 ("dev_slab_layout", C.c_int32), ("host_slab_layout", C.c_int32), ("staging_slots", C.c_int32),
                 ("host_threads", C.c_int32), ("kernel", C.c_int32), ("migrate_ctas", C.c_int32),
                 ("flags", C.c_uint32), ("numa_node", C.c_int32), ("dma_piece_mib", C.c_uint32),
-                ("reserved", C.c_uint32 * 5)]
+                ("pack_layer_mib", C.c_uint32), ("reserved", C.c_uint32 * 4)]
 
 
 class WeightDesc(C.Structure):

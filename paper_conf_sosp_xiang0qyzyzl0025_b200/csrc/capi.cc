@@ -118,6 +118,7 @@ int aeg_config_default(aeg_config* cfg) {
     cfg->host_slab_layout = AEG_LAYER_MAJOR;
     cfg->kernel = AEG_KERNEL_AUTO;
     cfg->dma_piece_mib = 128;
+    cfg->pack_layer_mib = 32;  // per-request swaps of small layers (bench per_request_sync)
     return AEG_OK;
   });
 }
@@ -137,6 +138,7 @@ int aeg_init(int device, const aeg_config* cfg, aeg_ctx* out) {
     if (!c.table_arena_bytes) c.table_arena_bytes = d.table_arena_bytes;
     if (!c.host_threads) c.host_threads = d.host_threads;
     if (!c.dma_piece_mib) c.dma_piece_mib = d.dma_piece_mib;
+    if (!c.pack_layer_mib) c.pack_layer_mib = d.pack_layer_mib;
     auto* x = new aeg_ctx_s();
     try {
       x->c.init(device, c);

@@ -18,23 +18,22 @@ namespace aeg {
 
 namespace {
 
-constexpr uint64_t kPackLayerBytes = 4ull << 20;  // layers smaller than this share a segment
-
 struct Seg {
   int32_t la, lb, i0, i1;
 };
 
 // A transfer of n blocks x L layers is cut into segments that fit one staging slot: whole layers
-// (several when a layer is tiny) or, for big layers, runs of blocks of one layer.  Segments are in
-// layer order, so the per-layer event can be recorded right after a layer's last segment.
-std::vector<Seg> plan(int32_t L, int32_t n, uint64_t chunk, uint64_t slot_bytes) {
+// (several when a layer is smaller than pack_bytes, aeg_config.pack_layer_mib) or, for big layers,
+// runs of blocks of one layer.  Segments are in layer order, so the per-layer event can be recorded
+// right after a layer's last segment.
+std::vector<Seg> plan(int32_t L, int32_t n, uint64_t chunk, uint64_t slot_bytes, uint64_t pack_bytes) {
   std::vector<Seg> out;
   if (n == 0) return out;
   const uint64_t layer = uint64_t(n) * chunk;
   if (layer <= slot_bytes) {
     int32_t lps = 1;
-    if (layer < kPackLayerBytes)
-      lps = int32_t(std::max<uint64_t>(1, std::min<uint64_t>(kPackLayerBytes, slot_bytes) / layer));
+    if (layer < pack_bytes)
+      lps = int32_t(std::max<uint64_t>(1, std::min<uint64_t>(pack_bytes, slot_bytes) / layer));
     lps = std::min(lps, L);
     for (int32_t la = 0; la < L; la += lps) out.push_back({la, std::min(L, la + lps), 0, n});
   } else {
@@ -319,7 +318,7 @@ uint64_t Ctx::swap_out(const Shape& sh, const aeg_block* dev, const aeg_block* h
     fetch_table(dtab, htab, uint64_t(n) * 8, s_gather);
   }
   pc.lap(2);
-  const auto segs = plan(sh.L, n, sh.chunk(), ring_out.slot_bytes);
+  const auto segs = plan(sh.L, n, sh.chunk(), ring_out.slot_bytes, uint64_t(cfg.pack_layer_mib) << 20);
   const auto runs = runs_of(host, n);
   const uint64_t dstride = dp.lstride(sh);
   const uint64_t piece_bytes = uint64_t(cfg.dma_piece_mib) << 20;
@@ -489,7 +488,7 @@ uint64_t Ctx::swap_in_from(const Shape& sh, int32_t peer, const aeg_block* host,
     // a ring slot, profiles/r01/timeline.txt; and no H2D copy queued behind other transfers' DMAs)
     fetch_table(dtab, htab, uint64_t(n) * 8, s_scatter);
   }
-  const auto segs = plan(sh.L, n, sh.chunk(), ring_in.slot_bytes);
+  const auto segs = plan(sh.L, n, sh.chunk(), ring_in.slot_bytes, uint64_t(cfg.pack_layer_mib) << 20);
   const auto runs = runs_of(host, n);
   const uint64_t dstride = dp.lstride(sh);
   const uint64_t piece_bytes = uint64_t(cfg.dma_piece_mib) << 20;
@@ -636,7 +635,7 @@ uint64_t Ctx::migrate(const Shape& sh, const aeg_block* src, int32_t peer, const
       for (int32_t i = 0; i < n; ++i) t[i] = dp.off0(src[i], sh);
       fetch_table(dtab, htab, uint64_t(n) * 8, s_gather);
     }
-    const auto segs = plan(sh.L, n, sh.chunk(), ring_out.slot_bytes);
+    const auto segs = plan(sh.L, n, sh.chunk(), ring_out.slot_bytes, uint64_t(cfg.pack_layer_mib) << 20);
     const auto runs = runs_of(dst, n);
     const uint64_t sstride = dp.lstride(sh);
     for (const Seg& g : segs) {

@@ -85,7 +85,7 @@ def test_after_covers_blocks_it_did_not_write():
                              dev_slab_layout=aeg.BLOCK_MAJOR, host_slab_layout=aeg.LAYER_MAJOR,
                              staging_slot_bytes=8 << 20, staging_slots=3, stage_ring_bytes=4 << 20,
                              stage_chunk_bytes=1 << 20, device_weight_bytes=8 << 20, table_arena_bytes=4 << 20,
-                             host_threads=2, kernel=aeg.KERNEL_AUTO, dma_piece_mib=1)
+                             host_threads=2, kernel=aeg.KERNEL_AUTO, dma_piece_mib=1, pack_layer_mib=1)
     ctx = aeg.Context(0, cfg)
     dev = Side(ctx, aeg.POOL_DEVICE, cfg.device_kv_bytes, cfg.dev_slab_bytes, aeg.BLOCK_MAJOR)
     host = Side(ctx, aeg.POOL_HOST, cfg.host_kv_bytes, cfg.host_slab_bytes, aeg.LAYER_MAJOR)
@@ -108,6 +108,8 @@ def test_after_covers_blocks_it_did_not_write():
             hc, ho = host.alloc(SHP, len(o))
             xs.append(ctx.kv_swap_out(SHP.as_tuple(), c, hc))
             hosts.append((hc, ho))
+        # X2 really ran its D2H in pieces (its transfer blob carries the piece table and events)
+        assert len(ctx.xfer_export(xs[1])) > 40 + (SHP.L + 1) * 64
         # read 64 of X1's host blocks only, ordered through `after` = X2 (X2 wrote none of them)
         rng = np.random.default_rng(5)
         pick = sorted(rng.choice(256, size=64, replace=False).tolist())

@@ -281,7 +281,7 @@ def test_two_process_host_route_p_c_d(nblocks):
                                  host_slab_bytes=MIB, host_slab_layout=aeg.BLOCK_MAJOR, staging_slot_bytes=MIB,
                                  staging_slots=2, stage_ring_bytes=4 * MIB, stage_chunk_bytes=MIB,
                                  table_arena_bytes=2 * MIB, host_threads=1, flags=aeg.CFG_SHARED_HOST,
-                                 dma_piece_mib=1)
+                                 dma_piece_mib=1, pack_layer_mib=1)
         a = aeg.Context(0, cfg)
         A = Side(a, aeg.POOL_DEVICE, nslabs * MIB, MIB, aeg.LAYER_MAJOR)
         H = Side(a, aeg.POOL_HOST, nslabs * MIB, MIB, aeg.BLOCK_MAJOR)

@@ -51,7 +51,7 @@ def test_random_overlapping_transfers_with_d2h_pieces(seed):
                              host_slab_layout=(seed // 2) % 2, staging_slot_bytes=(4 << 20) if seed % 2 else (8 << 20),
                              staging_slots=2, stage_ring_bytes=4 << 20, stage_chunk_bytes=1 << 20,
                              device_weight_bytes=2 << 20, table_arena_bytes=2 << 20, host_threads=1,
-                             kernel=aeg.KERNEL_AUTO, dma_piece_mib=1)
+                             kernel=aeg.KERNEL_AUTO, dma_piece_mib=1, pack_layer_mib=1)
     log, n_out = _stress(100 + seed, cfg, SHB, 28, lo=14)
     # the swap-outs really ran in pieces: more D2H ops than (swap-out, layer) pairs
     assert n_out > 0 and sum(1 for e in log if e[0] == "op" and e[1] == "d2h") > n_out * SHB.L

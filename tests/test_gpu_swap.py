@@ -171,7 +171,7 @@ def test_swap_in_waits_per_d2h_piece(host_layout, slot):
                              dev_slab_layout=aeg.LAYER_MAJOR, host_slab_layout=host_layout,
                              staging_slot_bytes=slot, staging_slots=3, stage_ring_bytes=4 << 20,
                              stage_chunk_bytes=1 << 20, device_weight_bytes=8 << 20, table_arena_bytes=4 << 20,
-                             host_threads=2, kernel=aeg.KERNEL_AUTO, dma_piece_mib=1)
+                             host_threads=2, kernel=aeg.KERNEL_AUTO, dma_piece_mib=1, pack_layer_mib=1)
     ctx = aeg.Context(0, cfg)
     dev = Side(ctx, aeg.POOL_DEVICE, cfg.device_kv_bytes, cfg.dev_slab_bytes, aeg.LAYER_MAJOR)
     host = Side(ctx, aeg.POOL_HOST, cfg.host_kv_bytes, cfg.host_slab_bytes, host_layout)
@@ -233,7 +233,7 @@ def test_swap_in_from_two_piecewise_swap_outs():
                              dev_slab_layout=aeg.BLOCK_MAJOR, host_slab_layout=aeg.LAYER_MAJOR,
                              staging_slot_bytes=8 << 20, staging_slots=3, stage_ring_bytes=4 << 20,
                              stage_chunk_bytes=1 << 20, device_weight_bytes=8 << 20, table_arena_bytes=4 << 20,
-                             host_threads=2, kernel=aeg.KERNEL_AUTO, dma_piece_mib=1)
+                             host_threads=2, kernel=aeg.KERNEL_AUTO, dma_piece_mib=1, pack_layer_mib=1)
     ctx = aeg.Context(0, cfg)
     dev = Side(ctx, aeg.POOL_DEVICE, cfg.device_kv_bytes, cfg.dev_slab_bytes, aeg.BLOCK_MAJOR)
     host = Side(ctx, aeg.POOL_HOST, cfg.host_kv_bytes, cfg.host_slab_bytes, aeg.LAYER_MAJOR)
