@@ -14,9 +14,12 @@ untouched.  bench.py runs the oracle (oracle/) only in its cpu_baseline leg and 
 the oracle parity of the same workloads is in tests/ (test_gpu_fullsize.py, test_gpu_c5.py).
 
 Also measured in the same run (not in `value`): H7+H8 model switch among Qwen-1.8B / Llama-7B /
-Yi-9B shapes with 1 GiB KV each (configs[3]), H5 local migrate (configs[2] shapes, one GPU), the
-oracle on host cores (cpu_baseline), and the whole step through the public Python API with
-wall-clock timing (e2e).
+Yi-9B shapes with 1 GiB KV each (configs[3]; staged, registered-cache and prefetch modes, Eq. 4 beta),
+H5 hand-off (configs[2] shapes: fused kernel, copy-engine route, per-chunk memcpy baseline; across
+GPUs at N >= 2), the P->C->D host route, configs[4] TP=4 scale-up, per-layer overlap, per-request
+sync overhead (Fig. 15 right), small-chunk shapes, configs[0] latency, the allocator, NVML PCIe
+counters, the oracle on host cores (cpu_baseline), and the whole step through the public Python
+API with wall-clock timing (e2e).
 
     python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference]
 N > 1 runs under torchrun (one rank per GPU): every rank swaps its own batch (replicas, weak
