@@ -184,6 +184,8 @@ def test_error_codes_and_validation():
     assert c.kernel_stats(aeg.K_FETCH)[0] == 0
     cfg = aeg.default_config()
     assert cfg.dma_piece_mib == 128                      # sub-layer D2H pieces on by default
+    assert cfg.pack_layer_mib == 32                      # layers < 32 MiB share a staging segment
+    assert cfg.device_kv_bytes == 0                      # sized at init: 90 % of free VRAM (reading 22)
     c.shutdown()
 
 
