@@ -78,6 +78,8 @@ def parse():
     p.add_argument("--dma-piece-mib", type=int, default=0, help="swap-out D2H piece (0 = library default)")
     p.add_argument("--profile", action="store_true", help="short run for ncu (no side legs)")
     p.add_argument("--two-device-probe", action="store_true", help=argparse.SUPPRESS)
+    p.add_argument("--leg-budget-s", type=float, default=1500.0,
+                   help="wall-clock budget of the side legs after the timed region")
     return p.parse_args()
 
 
@@ -2003,6 +2005,53 @@ def run_ours(args):
     g_ms = g[2] / max(1, g[0])
     g_ach = g_per_launch_bytes / (g_ms * 1e6) if g_ms > 0 else 0.0
     s_ach = (s[1] / max(1, s[0])) / ((s[2] / max(1, s[0])) * 1e6) if s[2] > 0 else 0.0
+    core = {
+        "metric": METRIC, "value": round(value, 2), "unit": "GB/s", "n_gpus": world, "steps": args.steps,
+        "warmup": args.warmup, "ms_per_step": round(ms_step, 2),
+        "step_ms_p10_p50_p90": [pct(0.1), pct(0.5), pct(0.9)], "higher_is_better": True, "scaling": "weak",
+        "vs_baseline": None, "dtype": "bf16", "data": "synthetic",
+        "config": {"workload": "configs[1]: Qwen-7B-shaped KV (32 layers, 32 KV heads, d=128, bf16, 16-token "
+                               f"blocks), {n_req}-request decode batch swapped out and back in per step",
+                   "requests": n_req, "requests_per_rank": n_req,
+                   "requests_note": (None if n_req == args.requests else
+                                     f"reduced from {args.requests} per rank so that {world} ranks' pinned "
+                                     "host pools fit this node's RAM; per-rank work differs from N=1"),
+                   "tokens": int(sum(sb.lens)), "blocks": sb.n,
+                   "bytes_per_direction": sb.n * sb.sh.block_bytes(), "slab": "1 GiB layer-major",
+                   "placement": "device pool aged by seeded churn", "l2": "inputs larger than L2 (32 GiB/step)",
+                   "kernel": args.kernel, "staging_slot_mib": sb.cfg.staging_slot_bytes >> 20,
+                   "dma_piece_mib": sb.cfg.dma_piece_mib,
+                   "staging_slots": sb.cfg.staging_slots, "parallelism": f"replicas x{world}"},
+        "roofline": {"bound": "hbm", "kernel": "gather (swap-out, H2)", "achieved": round(g_ach, 1),
+                     "peak": hbm, "peak_source": hbm_src, "unit": "GB/s",
+                     "frac": round(g_ach / hbm, 3), "traffic": ncu_traffic("gather", int(g_per_launch_bytes)),
+                     "algorithmic_bytes_per_launch": int(g_per_launch_bytes), "launches": g[0],
+                     "mean_launch_ms": round(g_ms, 4), "scatter_achieved": round(s_ach, 1)},
+        "pcie": {"bound": "pcie", "achieved_round_trip": round(bytes_step / (ms_step * 1e6), 1),
+                 "achieved_per_direction": round(bytes_step / 2 / (ms_step * 1e6), 1),
+                 "peak_per_direction_nominal": PCIE_NOMINAL,
+                 "frac_of_duplex_nominal": round(bytes_step / (ms_step * 1e6) / (2 * PCIE_NOMINAL), 3)},
+        "clocks": clocks,
+        "pcie_counters": pcie_counters,
+        "gpu_launches": launches_all,
+        "consumer_launches": args.steps * sb.L,
+    }
+    # Side legs are bounded: a hung leg must not lose the headline line, so after leg_budget_s a
+    # watchdog prints the core line with the legs completed so far and ends the process.
+    import threading
+    partial, print_lock, printed = {}, threading.Lock(), []
+
+    def on_leg_timeout():
+        with print_lock:
+            if rank == 0 and not printed:
+                line = dict(core)
+                line.update({"side_legs_timed_out_after_s": args.leg_budget_s, "side_legs_completed": partial})
+                print(json.dumps(line), flush=True)
+                printed.append(1)
+        os._exit(0)
+    watchdog = threading.Timer(args.leg_budget_s, on_leg_timeout)
+    watchdog.daemon = True
+    watchdog.start()
     out = {}
     if not args.profile:
         pc = pcie_calibration(torch)
@@ -2029,14 +2078,17 @@ def run_ours(args):
                    "swap_out_layer0_landed_ms_p50": round(statistics.median(f[2] for f in fl), 2),
                    "enqueue_ms_p50": {"swap_out": round(statistics.median(f[3] for f in fl), 2),
                                       "swap_in": round(statistics.median(f[4] for f in fl), 2)}}
+        partial["e2e"] = e2e
         def leg(name, fn):
             """A side leg that fails reports its error in the line instead of losing the whole line."""
             try:
-                return fn()
+                r = fn()
             except Exception as e:  # noqa: BLE001
                 import traceback
                 log(f"[rank {rank}] leg {name} failed:\n" + traceback.format_exc())
-                return {"error": f"{type(e).__name__}: {e}"}
+                r = {"error": f"{type(e).__name__}: {e}"}
+            partial[name] = r
+            return r
 
         one_dir = leg("one_direction", lambda: sb.one_direction(torch, cons))
         ver = leg("verify", sb.verify)
@@ -2118,37 +2170,7 @@ def run_ours(args):
     else:
         sb.ctx.shutdown()
     if rank == 0:
-        res = {
-            "metric": METRIC, "value": round(value, 2), "unit": "GB/s", "n_gpus": world, "steps": args.steps,
-            "warmup": args.warmup, "ms_per_step": round(ms_step, 2),
-            "step_ms_p10_p50_p90": [pct(0.1), pct(0.5), pct(0.9)], "higher_is_better": True, "scaling": "weak",
-            "vs_baseline": None, "dtype": "bf16", "data": "synthetic",
-            "config": {"workload": "configs[1]: Qwen-7B-shaped KV (32 layers, 32 KV heads, d=128, bf16, 16-token "
-                                   f"blocks), {n_req}-request decode batch swapped out and back in per step",
-                       "requests": n_req, "requests_per_rank": n_req,
-                       "requests_note": (None if n_req == args.requests else
-                                         f"reduced from {args.requests} per rank so that {world} ranks' pinned "
-                                         "host pools fit this node's RAM; per-rank work differs from N=1"),
-                       "tokens": int(sum(sb.lens)), "blocks": sb.n,
-                       "bytes_per_direction": sb.n * sb.sh.block_bytes(), "slab": "1 GiB layer-major",
-                       "placement": "device pool aged by seeded churn", "l2": "inputs larger than L2 (32 GiB/step)",
-                       "kernel": args.kernel, "staging_slot_mib": sb.cfg.staging_slot_bytes >> 20,
-                       "dma_piece_mib": sb.cfg.dma_piece_mib,
-                       "staging_slots": sb.cfg.staging_slots, "parallelism": f"replicas x{world}"},
-            "roofline": {"bound": "hbm", "kernel": "gather (swap-out, H2)", "achieved": round(g_ach, 1),
-                         "peak": hbm, "peak_source": hbm_src, "unit": "GB/s",
-                         "frac": round(g_ach / hbm, 3), "traffic": ncu_traffic("gather", int(g_per_launch_bytes)),
-                         "algorithmic_bytes_per_launch": int(g_per_launch_bytes), "launches": g[0],
-                         "mean_launch_ms": round(g_ms, 4), "scatter_achieved": round(s_ach, 1)},
-            "pcie": {"bound": "pcie", "achieved_round_trip": round(bytes_step / (ms_step * 1e6), 1),
-                     "achieved_per_direction": round(bytes_step / 2 / (ms_step * 1e6), 1),
-                     "peak_per_direction_nominal": PCIE_NOMINAL,
-                     "frac_of_duplex_nominal": round(bytes_step / (ms_step * 1e6) / (2 * PCIE_NOMINAL), 3)},
-            "clocks": clocks,
-            "pcie_counters": pcie_counters,
-            "gpu_launches": launches_all,
-            "consumer_launches": args.steps * sb.L,
-        }
+        res = json.loads(json.dumps(core))
         res.update(out)
         pm = out.get("pcie_memcpy_GBps") or {}
         if pm.get("bidir_total"):   # the round trip against this box's own duplex copy-engine ceiling
@@ -2160,7 +2182,11 @@ def run_ours(args):
             res["pcie"]["swap_in_alone_GBps"] = od["swap_in"]["GBps"]
             res["pcie"]["swap_out_alone_frac"] = round(od["swap_out"]["GBps"] / PCIE_NOMINAL, 3)
             res["pcie"]["swap_in_alone_frac"] = round(od["swap_in"]["GBps"] / PCIE_NOMINAL, 3)
-        print(json.dumps(res), flush=True)
+        with print_lock:
+            if not printed:
+                print(json.dumps(res), flush=True)
+                printed.append(1)
+    watchdog.cancel()
     dist.close()
     return 0
 
