@@ -22,6 +22,8 @@ OBJ_DIR = os.path.join(ROOT, "build", "obj")
 
 CXXFLAGS = ["-O2", "-g", "-fPIC", "-std=c++17", "-Wall", "-Wno-unused-function", "-pthread"]
 NVFLAGS = ARCH + ["-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC", "-Xptxas", "-v"]
+# experiments only (tools/*.sh): extra -D flags for the kernels, e.g. "-DAEG_BW_GRID=120"
+NVFLAGS += os.environ.get("AEG_NVCC_EXTRA", "").split()
 
 
 def _needs(out: str, deps: list[str]) -> bool:

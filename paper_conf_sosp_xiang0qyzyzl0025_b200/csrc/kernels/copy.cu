@@ -353,7 +353,10 @@ cudaError_t launch_t(const CopyArgs& a, int impl, int max_ctas, cudaStream_t s) 
     const uint32_t cap = std::min<uint32_t>(16u << 10, uint32_t(kBwSmem / kBwWarps / 2) & ~15u);
     const uint32_t piece = a.chunk <= cap ? uint32_t(a.chunk) : cap;
     const uint64_t items = uint64_t(a.nl) * a.n * ((a.chunk + piece - 1) / piece);
-    uint64_t grid = max_ctas > 0 ? uint64_t(max_ctas) : uint64_t(kSMs);
+#ifndef AEG_BW_GRID
+#define AEG_BW_GRID kSMs
+#endif
+    uint64_t grid = max_ctas > 0 ? uint64_t(max_ctas) : uint64_t(AEG_BW_GRID);
     const uint64_t need = (items + kBwWarps - 1) / kBwWarps;  // one item per warp at least
     if (grid > need) grid = need;
     copy_bulkw<SP, DP><<<unsigned(grid), kBwWarps * 32, kBwSmem, s>>>(a, piece);
