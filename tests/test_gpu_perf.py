@@ -1,0 +1,52 @@
+"""Performance floor (not parity): the gather / scatter kernels of a swap must stay HBM-bound —
+at least 0.70 of the measured copy peak (north star target; they run at ~0.9–0.97), timed by the
+library's own CUDA events (AEG_CFG_TIMING) on 1 GiB per direction (one launch each way), for
+256 KiB (Qwen-7B) and 8 KiB (Yi-9B TP=4 rank) chunks.  PCIe rates are not asserted: they vary by box."""
+import json
+import os
+
+import pytest
+
+import paper_conf_sosp_xiang0qyzyzl0025_b200 as aeg
+
+from .gpu_harness import require_gpu
+
+pytestmark = pytest.mark.gpu
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+GIB = 1 << 30
+
+
+def _peak():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    return float(json.load(open(p))["hbm_gbs"]) if os.path.exists(p) else 6650.0
+
+
+@pytest.mark.parametrize("shape", [(32, 32, 128, 2, 16), (48, 1, 128, 2, 16)], ids=["256KiB", "8KiB"])
+def test_swap_kernels_stay_hbm_bound(shape):
+    require_gpu()
+    sh = aeg.KVShape.of(shape)
+    n = GIB // sh.block_bytes()
+    # pack every layer into one 1 GiB segment: one gather and one scatter launch per transfer, so the
+    # events time the kernel body rather than per-launch overhead
+    ctx = aeg.Context(0, aeg.default_config(device_kv_bytes=4 * GIB, host_kv_bytes=2 * GIB,
+                                            pack_layer_mib=1024, flags=aeg.CFG_TIMING))
+    try:
+        dev = ctx.kv_alloc(aeg.POOL_DEVICE, shape, n)
+        for _ in range(3):   # warm-up rounds, then measure the last
+            ctx.kernel_stats_reset()
+            host = ctx.kv_alloc(aeg.POOL_HOST, shape, n)
+            x = ctx.kv_swap_out(shape, dev, host, flags=aeg.FREE_SRC)
+            ctx.layer_ready(x, -1, aeg.READY_BLOCK)
+            dev = ctx.kv_alloc(aeg.POOL_DEVICE, shape, n)
+            y = ctx.kv_swap_in(shape, host, dev, flags=aeg.FREE_SRC)
+            ctx.layer_ready(y, -1, aeg.READY_BLOCK)
+            ctx.xfer_release(x)
+            ctx.xfer_release(y)
+        floor = 0.70 * _peak()
+        for kind, name in ((aeg.K_GATHER, "gather"), (aeg.K_SCATTER, "scatter")):
+            launches, nbytes, ms = ctx.kernel_stats(kind)
+            assert launches > 0 and ms > 0
+            gbps = nbytes / (ms * 1e6)
+            assert gbps >= floor, f"{name}: {gbps:.0f} GB/s < {floor:.0f} (0.70 of the measured copy peak)"
+    finally:
+        ctx.shutdown()
