@@ -1786,6 +1786,37 @@ def overlap_leg(aeg, torch, kernel, work_us=500, reps=5, pack_mib=0):
     return out
 
 
+def kernel_alone_leg(aeg, kernel, shape=None):
+    """The dominant kernels without the step's concurrent PCIe DMA: one 1 GiB swap-out and swap-in of
+    the C2 shape with every layer in one staging segment (pack_layer_mib = 1024), i.e. one gather and
+    one scatter launch, timed by the library's CUDA events (AEG_CFG_TIMING); best of 3."""
+    shape = shape or QWEN7B
+    sh = aeg.KVShape.of(shape)
+    n = GIB // sh.block_bytes()
+    ctx = aeg.Context(0, aeg.default_config(device_kv_bytes=4 * GIB, host_kv_bytes=2 * GIB, pack_layer_mib=1024,
+                                            kernel=kernel, flags=aeg.CFG_TIMING))
+    best = {}
+    try:
+        dev = ctx.kv_alloc(aeg.POOL_DEVICE, shape, n)
+        for _ in range(4):
+            ctx.kernel_stats_reset()
+            host = ctx.kv_alloc(aeg.POOL_HOST, shape, n)
+            x = ctx.kv_swap_out(shape, dev, host, flags=aeg.FREE_SRC)
+            ctx.layer_ready(x, -1, aeg.READY_BLOCK)
+            dev = ctx.kv_alloc(aeg.POOL_DEVICE, shape, n)
+            y = ctx.kv_swap_in(shape, host, dev, flags=aeg.FREE_SRC)
+            ctx.layer_ready(y, -1, aeg.READY_BLOCK)
+            ctx.xfer_release(x)
+            ctx.xfer_release(y)
+            for kind, name in ((aeg.K_GATHER, "gather"), (aeg.K_SCATTER, "scatter")):
+                nl, nb, ms = ctx.kernel_stats(kind)
+                if ms > 0:
+                    best[name] = max(best.get(name, 0.0), nb / (ms * 1e6))
+    finally:
+        ctx.shutdown()
+    return {k: round(v, 1) for k, v in best.items()}
+
+
 def per_request_sync_leg(aeg, torch, kernel, h2d_GBps=None, n_req=32, pack_mib=0):
     """Fig. 15 (right) on B200: the per-request KV cache transfer overhead.  n_req
     Qwen-7B requests with ShareGPT-like lengths (lognormal prompt + output, seeded) sit in the host
@@ -2143,6 +2174,7 @@ def run_ours(args):
                   "model_cache_gen_s": round(gen_s, 1)}
             del caches
         ovl = None if args.no_switch or world > 1 else leg("overlap", lambda: overlap_leg(aeg, torch, kernel))
+        alone = leg("kernel_alone", lambda: kernel_alone_leg(aeg, kernel))
         prs = None if world > 1 else leg("per_request_sync", lambda: per_request_sync_leg(
             aeg, torch, kernel, h2d_GBps=pc.get("h2d")))
         if args.no_c5:
@@ -2160,6 +2192,7 @@ def run_ours(args):
         cpu = None if args.no_cpu or rank != 0 else leg("cpu_baseline", cpu_baseline)
         out.update({"e2e": e2e, "verify": ver, "one_direction": one_dir, "pcie_memcpy_GBps": {k: round(v, 1) for k, v in pc.items()},
                     "switch": sw, "migrate": mig, "per_layer_overlap": ovl, "per_request_sync": prs, "c5": c5,
+                    "kernel_alone": alone,
                     "allocator": alloc,
                     "per_chunk_memcpy_baseline": base, "small_chunk": small, "small_chunk_tp4": small_tp4, "c1": c1, "back_to_back": back2back,
                     "host_route": route,
@@ -2172,6 +2205,11 @@ def run_ours(args):
     if rank == 0:
         res = json.loads(json.dumps(core))
         res.update(out)
+        ka = out.get("kernel_alone") or {}
+        if ka.get("gather"):   # context: the same kernel with no concurrent DMA (one 1 GiB launch)
+            res["roofline"]["alone_achieved"] = ka["gather"]
+            res["roofline"]["alone_frac"] = round(ka["gather"] / hbm, 3)
+            res["roofline"]["alone_scatter_achieved"] = ka.get("scatter")
         pm = out.get("pcie_memcpy_GBps") or {}
         if pm.get("bidir_total"):   # the round trip against this box's own duplex copy-engine ceiling
             res["pcie"]["measured_bidir_memcpy_GBps"] = round(pm["bidir_total"], 1)
