@@ -24,6 +24,7 @@ CXXFLAGS = ["-O2", "-g", "-fPIC", "-std=c++17", "-Wall", "-Wno-unused-function",
 NVFLAGS = ARCH + ["-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC", "-Xptxas", "-v"]
 # experiments only (tools/*.sh): extra -D flags for the kernels, e.g. "-DAEG_BW_GRID=120"
 NVFLAGS += os.environ.get("AEG_NVCC_EXTRA", "").split()
+CXXFLAGS += os.environ.get("AEG_CXX_EXTRA", "").split()   # same, for the runtime (e.g. swap.cc)
 
 
 def _needs(out: str, deps: list[str]) -> bool:

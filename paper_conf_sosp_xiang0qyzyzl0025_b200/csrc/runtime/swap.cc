@@ -680,12 +680,18 @@ uint64_t Ctx::migrate(const Shape& sh, const aeg_block* src, int32_t peer, const
     if (flags & AEG_FREE_SRC) dp.free(src, n);
     return x->id;
   }
-  // Layers per launch: every launch pays a fixed ~8-36 us, so pack layers up to a
-  // target payload.  Same-device destinations copy at HBM speed (a 133 MiB layer is ~45 us): pack to
-  // 512 MiB.  Over NVLink a 128 MiB launch already takes ~170 us, and per-layer readiness lets the
-  // decode instance start early, so remote destinations keep (at least) one launch per 128 MiB.
+  // Layers per launch.  A launch boundary costs a fixed ~15 us (ramp + drain of the streaming
+  // pipeline; not hidden by a second kernel stream, whose concurrent CTAs lose as much to DRAM
+  // efficiency): one configs[2] hand-off (16 Llama-2-13B requests, 733 MiB per layer) takes 10.09 ms
+  // as 40 launches, 9.70 ms as 8 and 9.48 ms as 1 (profiles/r02/migrate_pack.txt).  So pack layers up
+  // to >= ~1 ms of copying per launch: 4 GiB on the same GPU (HBM speed), 512 MiB over NVLink
+  // (~0.7 ms at the measured 770 GB/s peer copy).  Every layer still gets its event, recorded when
+  // its launch completes; layers larger than the pack go one per launch.
+#ifndef AEG_MIGRATE_LOCAL_PACK_MIB  // overridable for experiments (tools/gpu_migrate_pack.sh)
+#define AEG_MIGRATE_LOCAL_PACK_MIB 4096
+#endif
   const bool remote = P && (!P->same_process || P->device != device);
-  const uint64_t pack = remote ? (128ull << 20) : (512ull << 20);
+  const uint64_t pack = remote ? (512ull << 20) : (uint64_t(AEG_MIGRATE_LOCAL_PACK_MIB) << 20);
   const uint64_t layer = uint64_t(n) * sh.chunk();
   int32_t lps = 1;
   if (n > 0 && layer < pack) lps = int32_t(std::min<uint64_t>(sh.L, std::max<uint64_t>(1, pack / layer)));

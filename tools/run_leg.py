@@ -1,5 +1,5 @@
 """Run one bench.py side leg alone on cuda:0 and print its JSON (development / profiling helper).
-    python tools/run_leg.py c5|migrate|overlap|small_chunk|switch|host_route [auto|lsu|bulk]"""
+    python tools/run_leg.py c5|migrate|overlap|small_chunk|switch|host_route|kernel_alone [auto|lsu|bulk]"""
 import json
 import os
 import sys
@@ -29,14 +29,15 @@ def switch_cmp(kernel):
 def main():
     build.build()
     leg = sys.argv[1]
-    kernel = {"auto": aeg.KERNEL_AUTO, "lsu": aeg.KERNEL_LSU, "bulk": aeg.KERNEL_BULK}[
+    kernel = {"auto": aeg.KERNEL_AUTO, "lsu": aeg.KERNEL_LSU, "bulk": aeg.KERNEL_BULK, "bulkw": aeg.KERNEL_BULKW}[
         sys.argv[2] if len(sys.argv) > 2 else "auto"]
     fn = {"c5": lambda: bench.c5_leg(aeg, torch, kernel),
           "migrate": lambda: bench.migrate_leg(aeg, torch, kernel),
           "overlap": lambda: bench.overlap_leg(aeg, torch, kernel),
           "small_chunk": lambda: bench.small_chunk_leg(aeg, torch, kernel),
           "switch": lambda: switch_cmp(kernel),
-          "host_route": lambda: bench.host_route_leg(aeg, torch, kernel)}[leg]
+          "host_route": lambda: bench.host_route_leg(aeg, torch, kernel),
+          "kernel_alone": lambda: bench.kernel_alone_leg(aeg, kernel)}[leg]
     print(json.dumps(fn()), flush=True)
 
 
