@@ -2,6 +2,7 @@
 // into an AEG_ERR_* code and a thread-local message; nothing throws across the ABI.
 #include <unistd.h>
 
+#include <algorithm>
 #include <cstring>
 #include <mutex>
 #include <string>
@@ -613,8 +614,11 @@ int aeg_xfer_import(aeg_ctx ctx, int32_t peer, const void* buf, uint64_t len, ae
     XferBlobHead h;
     std::memcpy(&h, buf, sizeof h);
     AEG_REQUIRE(h.magic == kXferMagic, AEG_ERR_INVALID, "not an aegkv transfer blob");
-    AEG_REQUIRE(h.L >= 0 && h.npiece >= 0 && h.n >= 0 && len >= xfer_blob_bytes(h.L, h.npiece, h.n),
-                AEG_ERR_INVALID, "blob truncated");
+    // bounds first (a shape has at most 4096 layers, a piece at least one block), so the size
+    // arithmetic below cannot overflow on a malformed blob
+    AEG_REQUIRE(h.L >= 0 && h.L <= 4096 && h.n >= 0 && h.npiece >= 0 && h.npiece <= std::max(h.n, 1),
+                AEG_ERR_INVALID, "malformed transfer blob");
+    AEG_REQUIRE(len >= xfer_blob_bytes(h.L, h.npiece, h.n), AEG_ERR_INVALID, "blob truncated");
     const bool same = h.pid == int32_t(getpid());
     AEG_REQUIRE(same || h.ipc, AEG_ERR_INVALID, "transfer events are not interprocess-capable");
     std::lock_guard<std::mutex> g(c.mu);

@@ -294,3 +294,25 @@ def test_slab_size_must_keep_16_byte_alignment():
             aeg.Context(0, aeg.default_config(device_kv_bytes=3 * bad, host_kv_bytes=3 * SLAB, dev_slab_bytes=bad,
                                               host_slab_bytes=SLAB, flags=aeg.CFG_HOST_ONLY | aeg.CFG_NO_DAEMON))
         assert e.value.code == aeg.ERR_INVALID
+
+
+def test_malformed_transfer_blobs_are_rejected():
+    """aeg_xfer_import bounds the header before sizing the blob (no overflow on hostile values)."""
+    import os
+    import struct
+    ctx = aeg.Context(0, aeg.default_config(device_kv_bytes=1 << 30, host_kv_bytes=1 << 30,
+                                            flags=aeg.CFG_HOST_ONLY | aeg.CFG_NO_DAEMON))
+    try:
+        def blob(L, npiece, n, tail=0):
+            head = struct.pack("<IiiiQiiQ", 0xAE6A1BC2, os.getpid(), L, 0, 1, npiece, n, 1)
+            return head + bytes(tail)
+        for L, npiece, n in ((2 ** 31 - 1, 0, 0), (-1, 0, 0), (4097, 0, 0), (2, 5, 2), (2, 2 ** 31 - 1, 2 ** 31 - 1 - 1),
+                             (1, -3, 0), (1, 0, -1)):
+            with pytest.raises(aeg.AegError, match="malformed"):
+                ctx.xfer_import(0, blob(L, npiece, n, 4096))
+        with pytest.raises(aeg.AegError, match="truncated"):
+            ctx.xfer_import(0, blob(2, 0, 0, 64))          # needs 3 event handles
+        with pytest.raises(aeg.AegError, match="not an aegkv"):
+            ctx.xfer_import(0, b"\0" * 256)
+    finally:
+        ctx.shutdown()
