@@ -685,13 +685,17 @@ def c1_leg(aeg, torch, kernel, reps=200):
             "reps": reps, "bit_exact": bad == 0}
 
 
-def pcie_calibration(torch):
-    """Plain cudaMemcpy of 1 GiB pinned <-> device: the copy engines' measured ceiling here."""
+def pcie_calibration(torch, dist=None):
+    """Plain cudaMemcpy of 1 GiB pinned <-> device: the copy engines' measured ceiling here.  With
+    several ranks every phase starts after a barrier, so all GPUs copy at once (the ceiling the
+    replicas share: PCIe switch uplinks, host DRAM)."""
+    sync = dist.barrier if dist is not None and dist.world > 1 else (lambda: None)
     h = torch.empty(GIB, dtype=torch.uint8, pin_memory=True)
     d = torch.empty(GIB, dtype=torch.uint8, device="cuda")
     out = {}
     s = new_stream(torch)
     for name, fn in (("h2d", lambda: d.copy_(h, non_blocking=True)), ("d2h", lambda: h.copy_(d, non_blocking=True))):
+        sync()
         with torch.cuda.stream(s):
             fn()
             e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
@@ -706,6 +710,7 @@ def pcie_calibration(torch):
     d2 = torch.empty(GIB, dtype=torch.uint8, device="cuda")
     s2 = new_stream(torch)
     torch.cuda.synchronize()
+    sync()
     e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     e0.record(s)
     s2.wait_event(e0)
@@ -719,6 +724,10 @@ def pcie_calibration(torch):
     e1.synchronize()
     out["bidir_total"] = 6 * GIB / (e0.elapsed_time(e1) * 1e6)
     del h, d, h2, d2
+    if dist is not None and dist.world > 1:   # all ranks at once: the aggregate the replicas can reach
+        out["bidir_total_all_ranks"] = dist.sum(out["bidir_total"])
+        out["h2d_all_ranks"] = dist.sum(out["h2d"])
+        out["d2h_all_ranks"] = dist.sum(out["d2h"])
     return out
 
 
@@ -740,6 +749,14 @@ def host_facts():
     except OSError:
         pass
     f["all_core_host_memcpy_GBps"] = host_memcpy_ceiling()
+    try:   # how the GPUs reach the host and each other (PCIe switches shared by GPUs bound the replicas)
+        r = subprocess.run(["nvidia-smi", "topo", "-m"], capture_output=True, text=True, timeout=30)
+        import re
+        f["nvidia_smi_topo"] = [" ".join(l.split()) for l in re.sub(r"\x1b\[[0-9;]*m", "", r.stdout).splitlines()
+                                if l.strip() and not l.lstrip().startswith(("Legend", "X ", "SYS", "NODE", "PHB",
+                                                                            "PXB", "PIX", "NV#"))][:20]
+    except (OSError, subprocess.SubprocessError):
+        pass
     return f
 
 
@@ -2025,6 +2042,8 @@ def run_ours(args):
         e1.synchronize()
     dist.barrier()
     ms_total = dist.max(e0.elapsed_time(e1))
+    # N > 1: each replica's own rate (the ranks share PCIe switch uplinks and host DRAM)
+    rank_ms = dist.gather_obj(e0.elapsed_time(e1)) if world > 1 else None
     clocks = clk.summary()
     pcie_counters = pcnt.summary()
     ms_step = ms_total / args.steps
@@ -2073,6 +2092,8 @@ def run_ours(args):
         "gpu_launches": launches_all,
         "consumer_launches": args.steps * sb.L,
     }
+    if rank_ms:
+        core["per_rank_GBps"] = [round(bytes_step * args.steps / (m * 1e6), 1) for m in rank_ms]
     # Side legs are bounded: a hung leg must not lose the headline line, so after leg_budget_s a
     # watchdog prints the core line with the legs completed so far and ends the process.
     import threading
@@ -2091,7 +2112,7 @@ def run_ours(args):
     watchdog.start()
     out = {}
     if not args.profile:
-        pc = pcie_calibration(torch)
+        pc = pcie_calibration(torch, dist)
         # e2e: the same step through the public Python API, wall clock, after a host sync each step
         e2e = None
         if not args.no_e2e:
@@ -2220,6 +2241,10 @@ def run_ours(args):
         if pm.get("bidir_total"):   # the round trip against this box's own duplex copy-engine ceiling
             res["pcie"]["measured_bidir_memcpy_GBps"] = round(pm["bidir_total"], 1)
             res["pcie"]["frac_of_measured_bidir"] = round(value / pm["bidir_total"], 3)
+        if pm.get("bidir_total_all_ranks"):   # N > 1: `value` is all ranks' bytes; ceiling = all GPUs at once
+            res["pcie"]["scope"] = "achieved_* and measured_bidir_memcpy_GBps: rank 0; *_all_ranks: every GPU at once"
+            res["pcie"]["measured_bidir_memcpy_GBps_all_ranks"] = round(pm["bidir_total_all_ranks"], 1)
+            res["pcie"]["frac_of_measured_bidir"] = round(value / pm["bidir_total_all_ranks"], 3)
         od = out.get("one_direction")
         if od and "error" not in od:   # each direction alone against PCIe Gen5 x16 nominal 64 GB/s (target >= 0.80)
             res["pcie"]["swap_out_alone_GBps"] = od["swap_out"]["GBps"]
