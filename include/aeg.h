@@ -260,6 +260,8 @@ int aeg_kv_swap_in(aeg_ctx ctx, const aeg_kv_shape* shape, const aeg_block* host
  * aeg_import_peer, or -1 for this context's own device pool (local relocation).  dst handles are
  * allocated by the peer in its device pool and are trusted (validated against the peer's
  * geometry only).  Per-layer events are interprocess-capable; export them with aeg_xfer_export.
+ * Consecutive layers share a kernel launch up to ~1 ms of copying (4 GiB on one GPU, 512 MiB to
+ * another GPU); each layer's event is recorded when the launch holding it completes.
  * AEG_FREE_SRC frees the source blocks.  AEG_MIGRATE_CE takes the copy-engine route (SURVEY H5
  * alternative): per staging segment a gather kernel packs the source blocks into the out staging
  * ring, then copy engines write the destination runs (one command per run and layer, or one 2-D
