@@ -78,6 +78,9 @@ def parse():
     p.add_argument("--dma-piece-mib", type=int, default=0, help="swap-out D2H piece (0 = library default)")
     p.add_argument("--profile", action="store_true", help="short run for ncu (no side legs)")
     p.add_argument("--two-device-probe", action="store_true", help=argparse.SUPPRESS)
+    p.add_argument("--probe-peer-bulk", action="store_true",
+                   help="N >= 2: also time cp.async.bulk stores into another GPU's memory (BULKW) in a throw-away "
+                        "process; off by default — AUTO never uses them, and a fault there would be an Xid on the box")
     p.add_argument("--leg-budget-s", type=float, default=1500.0,
                    help="wall-clock budget of the side legs after the timed region")
     return p.parse_args()
@@ -2183,8 +2186,9 @@ def run_ours(args):
                 mig["two_device_same_process"] = leg("migrate_two_device",
                                                      lambda: migrate_leg_two_device(aeg, torch, kernel))
                 # bulk copies (cp.async.bulk) storing into another GPU's memory are not relied on by
-                # AUTO; measure them in a throw-away process so a fault cannot touch this one
-                mig["two_device_bulkw_stores_probe"] = leg("two_device_bulkw", two_device_bulkw_probe)
+                # AUTO; opt-in only, and then in a throw-away process so a fault cannot touch this one
+                if args.probe_peer_bulk:
+                    mig["two_device_bulkw_stores_probe"] = leg("two_device_bulkw", two_device_bulkw_probe)
             dist.barrier()
         else:
             mig = leg("migrate", lambda: migrate_leg(aeg, torch, kernel, args.migrate_requests))
