@@ -2131,8 +2131,9 @@ def run_ours(args):
                           + sb.enqueue_ms)
             e2e_t = dist.max(statistics.median(ts))   # the job's step ends when the slowest rank's does
             e2e = {"value": round(dist.sum(bytes_step) / e2e_t / 1e9, 2), "unit": "GB/s",
-                   "h2d_bytes_per_step": int(bytes_step // 2 + 2 * sb.n * 8),
-                   "d2h_bytes_per_step": int(bytes_step // 2),
+                   # whole job, like `value` (every rank's copies)
+                   "h2d_bytes_per_step": int(dist.sum(bytes_step // 2 + 2 * sb.n * 8)),
+                   "d2h_bytes_per_step": int(dist.sum(bytes_step // 2)),
                    "how": "wall clock around the Python-API calls of one step incl. host sync",
                    "round_trip_layer0_ready_ms_p50": round(statistics.median(f[0] for f in fl), 2),
                    "round_trip_last_layer_ready_ms_p50": round(statistics.median(f[1] for f in fl), 2),
