@@ -124,6 +124,7 @@ struct WeightPipe {
   std::deque<std::unique_ptr<WJob>> jobs;
   std::deque<std::function<void()>> tasks;
   std::vector<uint8_t> filled;  // per chunk of the current job: parts filled so far
+  int64_t outstanding = 0;      // fill tasks queued or running (they point into the current job)
   static constexpr int kParts = 8;  // fill tasks per chunk (8 MiB each for 64 MiB chunks)
   bool stop = false;
   int nslots = 0;
@@ -181,12 +182,13 @@ struct WeightPipe {
     }
     if (ce > p) std::memset(dst + (p - cs), 0, ce - p);
     stream_fence();
-    bool done;
+    bool wake;
     {
       std::lock_guard<std::mutex> lk(m);
-      done = ++filled[ci] == parts;
+      wake = ++filled[ci] == parts;
+      wake = (--outstanding == 0) || wake;
     }
-    if (done) cv_filled.notify_all();
+    if (wake) cv_filled.notify_all();
   }
 
   void record_layers(WJob* j, const std::vector<uint64_t>& layer_last, uint64_t upto, cudaStream_t s) {
@@ -263,6 +265,7 @@ struct WeightPipe {
               std::lock_guard<std::mutex> lk(m);
               for (int part = 0; part < kParts; ++part)
                 tasks.push_back([this, j, q, slot, w, part] { fill(j, q, slot, w, part, kParts); });
+              outstanding += kParts;
             }
             cv_task.notify_all();
             ++dispatched;
@@ -288,8 +291,12 @@ struct WeightPipe {
         if (!j->x->recorded[l]) c->record(j->x, l, s);  // layers without tensors
       c->record(j->x, -1, s);
       c->w_inflight--;
-    } catch (const Error& e) {
+    } catch (const std::exception& e) {  // aeg::Error (CUDA failures) or host allocation failure
       fprintf(stderr, "aegkv: weight pipeline failed: %s\n", e.what());
+      {  // fill tasks already dispatched point into this job: let them finish before it is freed
+        std::unique_lock<std::mutex> lk(m);
+        cv_filled.wait(lk, [&] { return outstanding == 0; });
+      }
       cudaStreamSynchronize(s);
       (void)cudaGetLastError();
       std::lock_guard<std::mutex> g(c->mu);
