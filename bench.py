@@ -1806,7 +1806,15 @@ def overlap_leg(aeg, torch, kernel, work_us=500, reps=5, pack_mib=0):
     return out
 
 
-def kernel_alone_leg(aeg, kernel, shape=None, spread_gib=16):
+def kernel_alone_leg(aeg, kernel, shape=None):
+    """kernel_alone_once over blocks spread like the step's, plus the contiguous best case (SURVEY
+    §8(d): blocks allocated in order from a fresh pool)."""
+    out = kernel_alone_once(aeg, kernel, shape, spread_gib=16)
+    out["contiguous"] = kernel_alone_once(aeg, kernel, shape, spread_gib=0)
+    return out
+
+
+def kernel_alone_once(aeg, kernel, shape=None, spread_gib=16):
     """The dominant kernels without the step's concurrent PCIe DMA: one 1 GiB swap-out and swap-in of
     the C2 shape with every layer in one staging segment (pack_layer_mib = 1024), i.e. one gather and
     one scatter launch, timed by the library's CUDA events (AEG_CFG_TIMING); best of 3.  The blocks
@@ -1816,14 +1824,17 @@ def kernel_alone_leg(aeg, kernel, shape=None, spread_gib=16):
     shape = shape or QWEN7B
     sh = aeg.KVShape.of(shape)
     n = GIB // sh.block_bytes()
-    ctx = aeg.Context(0, aeg.default_config(device_kv_bytes=spread_gib * GIB, host_kv_bytes=2 * GIB,
+    ctx = aeg.Context(0, aeg.default_config(device_kv_bytes=max(spread_gib, 4) * GIB, host_kv_bytes=2 * GIB,
                                             pack_layer_mib=1024, kernel=kernel, flags=aeg.CFG_TIMING))
     best = {}
     try:
-        every = ctx.kv_alloc(aeg.POOL_DEVICE, shape, (spread_gib * GIB) // sh.block_bytes())
-        keep = gi.rng(47).permutation(len(every))
-        ctx.kv_free(aeg.POOL_DEVICE, every[np.sort(keep[n:])])
-        dev = every[np.sort(keep[:n])]
+        if spread_gib:
+            every = ctx.kv_alloc(aeg.POOL_DEVICE, shape, (spread_gib * GIB) // sh.block_bytes())
+            keep = gi.rng(47).permutation(len(every))
+            ctx.kv_free(aeg.POOL_DEVICE, every[np.sort(keep[n:])])
+            dev = every[np.sort(keep[:n])]
+        else:   # contiguous best case: a fresh pool, blocks in order (whole-slab runs per layer)
+            dev = ctx.kv_alloc(aeg.POOL_DEVICE, shape, n)
         for _ in range(4):
             ctx.kernel_stats_reset()
             host = ctx.kv_alloc(aeg.POOL_HOST, shape, n)
