@@ -1957,14 +1957,38 @@ class OracleSample:
                 "31 GiB/direction step")
 
 
+def gpu_local_cpus(index=0):
+    """Host cores on GPU `index`'s NUMA node (sysfs local_cpulist of its PCI device), or None."""
+    try:
+        r = subprocess.run(["nvidia-smi", "--query-gpu=pci.bus_id", "--format=csv,noheader", "-i", str(index)],
+                           capture_output=True, text=True, timeout=30)
+        bus = r.stdout.strip().lower()
+        if bus.count(":") == 2 and len(bus.split(":")[0]) == 8:   # 00000000:1B:00.0 -> 0000:1b:00.0
+            bus = bus[4:]
+        cpus = set()
+        for part in open(f"/sys/bus/pci/devices/{bus}/local_cpulist").read().strip().split(","):
+            a, _, b = part.partition("-")
+            cpus.update(range(int(a), int(b or a) + 1))
+        return cpus or None
+    except (OSError, ValueError, subprocess.SubprocessError):
+        return None
+
+
 class one_core:
-    """Pin this process to one host core for the oracle's timing (single-threaded)."""
+    """Pin this process to one host core for the oracle's timing (single-threaded, a
+    core on the GPU's NUMA node when sysfs says which)."""
 
     def __enter__(self):
         self.aff = os.sched_getaffinity(0) if hasattr(os, "sched_getaffinity") else None
         if self.aff:
-            os.sched_setaffinity(0, {min(self.aff)})
+            near = (gpu_local_cpus() or set()) & set(self.aff)
+            self.core = min(near or self.aff)
+            self.gpu_local = bool(near)
+            os.sched_setaffinity(0, {self.core})
         return self
+
+    def describe(self):
+        return {"core_id": getattr(self, "core", None), "on_gpu_numa_node": getattr(self, "gpu_local", None)}
 
     def __exit__(self, *a):
         if self.aff:
@@ -1975,14 +1999,14 @@ def cpu_baseline(blocks=512, min_s=10.0):
     """cpu_baseline leg of our arm: OracleSample timed for >= min_s seconds on one core."""
     o = OracleSample(blocks)
     reps, t = 0, 0.0
-    with one_core():
+    with one_core() as pin:
         while (reps == 0 or t < min_s) and reps < 50:
             t0 = time.perf_counter()
             o.rep()
             t += time.perf_counter() - t0
             reps += 1
     return {"value": round(o.bytes_per_rep() * reps / t / 1e9, 3), "unit": "GB/s", "cores": 1, "kind": "oracle",
-            "sample": o.describe(reps, t)}
+            "sample": o.describe(reps, t), "pinning": pin.describe()}
 
 
 # ----------------------------------------------------------------------------------- arms
@@ -1993,7 +2017,7 @@ def run_reference(args):
     if rank != 0:
         return 0
     o = OracleSample(512)
-    with one_core():
+    with one_core() as pin:
         for _ in range(args.warmup):
             o.rep()
         t = 0.0
@@ -2011,7 +2035,7 @@ def run_reference(args):
                                   f"{o.blocks} of {sum(c2_requests(args.requests)[1])} blocks per step)",
                       "requests": args.requests},
            "cpu_baseline": {"value": round(value, 3), "unit": "GB/s", "cores": 1, "kind": "oracle",
-                            "sample": o.describe(args.steps, t)},
+                            "sample": o.describe(args.steps, t), "pinning": pin.describe()},
            "e2e": {"value": round(value, 3), "unit": "GB/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(out), flush=True)
     return 0
