@@ -149,3 +149,22 @@ def test_migrate_is_relabelled_identity():
     hg = PoolGeom(2 * SLAB, SLAB, BLOCK_MAJOR)
     mid = kv.swap_out(src, sg, np.zeros(hg.nbytes, np.uint8), hg, SH, a, [(1, 1), (0, 0)])
     assert np.array_equal(kv.swap_in(mid, hg, dst, dg, SH, [(1, 1), (0, 0)], b), out)
+
+
+def test_oracle_functions_do_not_modify_their_inputs():
+    """O3-O7 are functions of their inputs (the returned image is the new state); the source and
+    destination arrays passed in stay exactly as they were."""
+    sh = KVShape(2, 1, 8, 2, 1)
+    g = PoolGeom(4 * sh.block_bytes(), 2 * sh.block_bytes(), LAYER_MAJOR)
+    r = np.random.default_rng(5)
+    src = r.integers(0, 256, g.nbytes, dtype=np.uint8)
+    dst = r.integers(0, 256, g.nbytes, dtype=np.uint8)
+    s0, d0 = src.copy(), dst.copy()
+    hs, hd = [(0, 0), (1, 1)], [(1, 0), (0, 1)]
+    out = kv.copy_blocks(src, g, dst, g, sh, hs, hd)
+    assert np.array_equal(src, s0) and np.array_equal(dst, d0)
+    assert not np.array_equal(out, d0)
+    stage = kv.gather(src, g, sh, hs, 0, sh.L)
+    assert np.array_equal(src, s0)
+    kv.scatter(dst, g, sh, hd, 0, sh.L, stage)
+    assert np.array_equal(dst, d0)

@@ -111,3 +111,22 @@ def test_record_captures_only_its_own_stream():
            ("wait", "C", "e"), ("use", "C", ["x"])]
     with pytest.raises(RuleViolation, match="❶"):
         check(bad)
+
+
+def test_ordering_is_transitive_through_another_stream():
+    """Table 2: a wait orders all future work of a stream after the captured work, so an order
+    established through an intermediate stream (P -> S -> D, no direct P -> D wait) holds: D may read
+    what P wrote.  Without the middle link the same read breaks rule ❷."""
+    cells = [("C", 0, 0)]
+    log = [
+        ("op", "P.kvout", "P->C", [], cells),
+        ("record", "P.kvout", "e1"),
+        ("wait", "S.aux", "e1"),
+        ("op", "S.aux", "unrelated", [], [("X", 0, 0)]),
+        ("record", "S.aux", "e2"),
+        ("wait", "D.kvin", "e2"),
+        ("op", "D.kvin", "C->D", cells, [("D", 0, 0)]),
+    ]
+    assert check(log)
+    with pytest.raises(RuleViolation, match="❷"):
+        check([e for e in log if e != ("wait", "S.aux", "e1")])

@@ -31,6 +31,13 @@ MUTANTS = [
     ("oracle/slab.py", "self.peak_assigned = max(self.peak_assigned, sum(v[0] for v in per.values()) * self.slab_bytes)", "self.peak_assigned = sum(v[0] for v in per.values()) * self.slab_bytes"),
     ("oracle/rules.py", "pending.setdefault(e[1], set()).add(c)", "pass"),
     ("oracle/rules.py", "captured[e[2]] = tail.get(e[1])", "captured[e[2]] = len(ops) - 1 if ops else None"),
+    ("oracle/rules.py", "            p.update(synced)\n", "            pass\n"),
+    ("oracle/rules.py", "            a |= anc[q]\n", "            pass\n"),
+    ("oracle/rules.py", "            if w is not None and w not in anc[i]:\n                rule", "            if False:\n                rule"),
+    ("oracle/rules.py", "for r in reads_since.get(c, ()):", "for r in ():"),
+    ("oracle/rules.py", "rule = \"❶\" if kind == \"use\" else \"❷\"", "rule = \"❷\""),
+    ("oracle/kv.py", "out = dst.copy()", "out = dst"),
+    ("oracle/kv.py", "    out = pool.copy()\n    n, c = len(handles), _c(sh, unit)", "    out = pool\n    n, c = len(handles), _c(sh, unit)"),
 ]
 
 
