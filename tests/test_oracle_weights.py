@@ -106,3 +106,24 @@ def test_region_exact_fit_and_one_byte_over():
     assert img.size == need and offs[-1] == last
     with pytest.raises(W.WeightError):
         W.stage(tens, descs, 0, 1, region_bytes=need - 1, base=base)
+
+
+def test_row_split_has_no_groups():
+    """Reading 18: `groups` cuts fused QKV-style tensors into row groups, so it applies to COL/VOCAB
+    only; a ROW (strided column) split with groups > 1 is undefined and rejected."""
+    w = np.zeros((6, 4, 2), np.uint8)
+    with pytest.raises(W.WeightError):
+        W.shard(w, W.ROW, 2, 0, 2)
+    with pytest.raises(W.WeightError):
+        W.shard(w, W.ROW, 3, 0, 1)
+
+
+def test_stage_leaves_the_given_image_untouched():
+    """stage() returns the new region image; the `dst` passed in (the previous image) is not written."""
+    descs = [dict(rows=4, cols=8, split=W.REPLICATED, groups=1)]
+    ts = [tensor(4, 8, 9)]
+    before = np.full(4096, 0xAB, np.uint8)
+    keep = before.copy()
+    out, offs, _ = W.stage(ts, descs, 0, 1, 4096, dst=before)
+    assert np.array_equal(before, keep)
+    assert np.array_equal(out[:64], ts[0].reshape(-1)) and np.all(out[64:] == 0xAB)

@@ -38,6 +38,13 @@ MUTANTS = [
     ("oracle/rules.py", "rule = \"❶\" if kind == \"use\" else \"❷\"", "rule = \"❷\""),
     ("oracle/kv.py", "out = dst.copy()", "out = dst"),
     ("oracle/kv.py", "    out = pool.copy()\n    n, c = len(handles), _c(sh, unit)", "    out = pool\n    n, c = len(handles), _c(sh, unit)"),
+    ("oracle/weights.py", "if rows % (groups * tp):", "if rows % tp:"),
+    ("oracle/weights.py", "if cols % tp or groups != 1:", "if cols % tp:"),
+    ("oracle/weights.py", "        dst = dst.copy()\n", "        pass\n"),
+    ("oracle/weights.py", "        offs.append(p)\n        p = align_up(p + n)", "        p = align_up(p + n)\n        offs.append(p)"),
+    ("oracle/kv.py", "    k = g.slab_bytes // sh.block_bytes()\n    assert", "    k = g.slab_bytes // sh.chunk_bytes()\n    assert"),
+    ("oracle/kv.py", "    stage = np.empty((l1 - l0) * n * c, dtype=pool.dtype)\n    for l in range(l0, l1):",
+     "    stage = np.empty((l1 - l0) * n * c, dtype=pool.dtype)\n    for l in range(l0, max(l0, l1 - 1)):"),
 ]
 
 
