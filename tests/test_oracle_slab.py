@@ -234,3 +234,16 @@ def test_fragmentation_empty_pool_and_slab_tail():
     assert p.fragmentation() == 0.0
     p.alloc(A, 1)            # assigned 256, used 128; the peak is still 768 -> 128/768
     assert p.fragmentation() == pytest.approx(128 / 768)
+
+
+def test_zero_block_request_is_a_no_op():
+    """An empty request (an instance with nothing to move) allocates nothing, claims no slab and is
+    not an error (include/aeg.h aeg_kv_alloc: "n == 0 is a no-op"); a negative count is invalid."""
+    sh = KVShape(2, 4, 64, 2, 16)
+    p = SlabPool(8 * sh.block_bytes() * 4, 8 * sh.block_bytes())
+    assert p.alloc(sh, 0) == []
+    per, free = p.stats()
+    assert per == {} and free == p.n_slabs
+    with pytest.raises(AllocError) as e:
+        p.alloc(sh, -1)
+    assert e.value.code == INVALID

@@ -45,6 +45,14 @@ MUTANTS = [
     ("oracle/kv.py", "    k = g.slab_bytes // sh.block_bytes()\n    assert", "    k = g.slab_bytes // sh.chunk_bytes()\n    assert"),
     ("oracle/kv.py", "    stage = np.empty((l1 - l0) * n * c, dtype=pool.dtype)\n    for l in range(l0, l1):",
      "    stage = np.empty((l1 - l0) * n * c, dtype=pool.dtype)\n    for l in range(l0, max(l0, l1 - 1)):"),
+    ("oracle/slab.py", "        self.reclaim()                              # reading 9", "        pass  # reading 9"),
+    ("oracle/slab.py", "if self.shape[s] is not None and not self.owned[s] and not any(q[0] == s for q in self.quarantine):",
+     "if self.shape[s] is not None and not self.owned[s]:"),
+    ("oracle/slab.py", "if xs <= self.done]", "if xs & self.done]"),
+    ("oracle/slab.py", "if j not in self.owned[s] or (s, j) in seen:", "if j not in self.owned[s]:"),
+    ("oracle/slab.py", "if x not in self.done and b in blocks}", "if b in blocks}"),
+    ("oracle/slab.py", "if n < 0 or self.k(shape) == 0:", "if n <= 0 or self.k(shape) == 0:"),
+    ("oracle/slab.py", "peak = self.peak_assigned_shape.get(shape, 0)", "peak = self.peak_assigned"),
 ]
 
 
