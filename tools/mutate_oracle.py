@@ -56,28 +56,36 @@ MUTANTS = [
 ]
 
 
-def main():
+def run_one(path, old, new):
+    """Apply one mutant in a private copy of oracle/ + tests/ and run the oracle pins there."""
+    with tempfile.TemporaryDirectory() as d:
+        for sub in ("oracle", "tests", "aeg_inputs"):
+            shutil.copytree(os.path.join(ROOT, sub), os.path.join(d, sub),
+                            ignore=shutil.ignore_patterns("__pycache__", "*.so"))
+        f = os.path.join(d, path)
+        src = open(f).read()
+        assert old in src, (path, old)
+        open(f, "w").write(src.replace(old, new, 1))
+        r = subprocess.run([sys.executable, "-m", "pytest", "-x", "-q", "-p", "no:cacheprovider",
+                            "tests/test_oracle_shape.py", "tests/test_oracle_slab.py", "tests/test_oracle_kv.py",
+                            "tests/test_oracle_weights.py", "tests/test_oracle_rules.py", "tests/test_oracle_memmove.py"],
+                           cwd=d, capture_output=True, text=True)
+        return r.returncode != 0
+
+
+def main(jobs=None):
+    import concurrent.futures as cf
+    jobs = jobs or max(1, min(16, os.cpu_count() or 1))
+    with cf.ThreadPoolExecutor(max_workers=jobs) as ex:
+        killed = list(ex.map(lambda m: run_one(*m), MUTANTS))
     survived = []
-    for path, old, new in MUTANTS:
-        with tempfile.TemporaryDirectory() as d:
-            for sub in ("oracle", "tests", "aeg_inputs"):
-                shutil.copytree(os.path.join(ROOT, sub), os.path.join(d, sub),
-                                ignore=shutil.ignore_patterns("__pycache__", "*.so"))
-            f = os.path.join(d, path)
-            src = open(f).read()
-            assert old in src, (path, old)
-            open(f, "w").write(src.replace(old, new, 1))
-            r = subprocess.run([sys.executable, "-m", "pytest", "-x", "-q", "-p", "no:cacheprovider",
-                                "tests/test_oracle_shape.py", "tests/test_oracle_slab.py", "tests/test_oracle_kv.py",
-                                "tests/test_oracle_weights.py", "tests/test_oracle_rules.py", "tests/test_oracle_memmove.py"],
-                               cwd=d, capture_output=True, text=True)
-            status = "killed" if r.returncode != 0 else "SURVIVED"
-            print(f"{status:9s} {path}: {new[:70]!r}")
-            if r.returncode == 0:
-                survived.append((path, new))
+    for (path, _, new), k in zip(MUTANTS, killed):
+        print(f"{'killed' if k else 'SURVIVED':9s} {path}: {new[:70]!r}")
+        if not k:
+            survived.append((path, new))
     print(f"{len(MUTANTS) - len(survived)}/{len(MUTANTS)} mutants killed")
     return 1 if survived else 0
 
 
 if __name__ == "__main__":
-    sys.exit(main())
+    sys.exit(main(int(sys.argv[1]) if len(sys.argv) > 1 else None))
