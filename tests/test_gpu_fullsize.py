@@ -166,6 +166,68 @@ def test_c3_full_size_handoff():
         b.shutdown()
 
 
+def test_packed_local_migrate_with_a_short_last_launch():
+    """Local hand-off launches pack consecutive layers up to 4 GiB (swap.cc): with 1.5 GiB layers
+    and L = 3 the layers go as [0, 2) + [2, 3) — a multi-layer launch and a short last one.  Every
+    chunk of the destination pool equals oracle O7 on chunk labels, and each layer is ready (its
+    event recorded when the launch holding it completes) with its bytes in place."""
+    require_gpu()
+    from oracle import kv as OK
+    from oracle.shape import KVShape
+    from oracle.slab import SlabPool
+    sht = (3, 8, 128, 2, 16)                 # Cl = 64 KiB, block = 192 KiB
+    sh = KVShape(*sht)
+    cl = sh.chunk_bytes()
+    n = (3 << 29) // cl                      # 1.5 GiB per layer
+    slab = 1 << 30
+    nslab = -(-n // (slab // sh.block_bytes())) + 1
+    seed = gi.kv_seed(7)
+    mk = lambda lay: aeg.Context(0, aeg.default_config(device_kv_bytes=nslab * slab, host_kv_bytes=1 << 30,  # noqa: E731
+                                                       dev_slab_bytes=slab, dev_slab_layout=lay,
+                                                       flags=aeg.CFG_TIMING))
+    a, b = mk(aeg.LAYER_MAJOR), mk(aeg.BLOCK_MAJOR)
+    try:
+        ga = OK.PoolGeom(nslab * slab, slab, aeg.LAYER_MAJOR)
+        gb = OK.PoolGeom(nslab * slab, slab, aeg.BLOCK_MAJOR)
+        oa, ob = SlabPool(ga.nbytes, slab), SlabPool(gb.nbytes, slab)
+        abase, _ = a.pool_region(0)
+        bbase, _ = b.pool_region(0)
+        D.fill_region(bbase, gb.nbytes, seed, gi.poison_key(gi.TAG_NEVER, 0))
+        cells = gb.nbytes // cl
+        blab = np.uint64(gi.poison_key(gi.TAG_NEVER, 0)) + np.arange(cells, dtype=np.uint64) * np.uint64(cl // 8)
+        alab = np.zeros(ga.nbytes // cl, dtype=np.uint64)
+        sc, so = a.kv_alloc(0, sht, n), oa.alloc(sh, n)
+        dc, do = b.kv_alloc(0, sht, n), ob.alloc(sh, n)
+        assert [aeg.decode_block(x)[1:] for x in sc] == list(so)
+        assert [aeg.decode_block(x)[1:] for x in dc] == list(do)
+        offs = np.array([OK.addr(ga, sh, h, l) for h in so for l in range(sh.L)], np.uint64)
+        keys = np.array([gi.kv_key(9, 0, j, l) for j in range(n) for l in range(sh.L)], np.uint64)
+        for i in range(0, offs.size, 1 << 16):
+            D.fill_chunks(abase, offs[i:i + (1 << 16)], keys[i:i + (1 << 16)], cl, seed)
+        alab[(offs // np.uint64(cl)).astype(np.int64)] = keys
+        a.import_peer(1, b.export_ipc())
+        a.kernel_stats_reset()
+        x = a.kv_migrate(sht, sc, 1, dc)
+        exp = OK.migrate(alab, ga, blab, gb, sh, so, do, unit=cl)
+        for l in range(sh.L):                # per-layer readiness: that layer's chunks are in place
+            a.layer_ready(x, l, aeg.READY_BLOCK)
+            lo = np.array([OK.addr(gb, sh, h, l) for h in do], np.uint64)
+            bad, _ = D.verify_chunks(bbase, lo, exp[(lo // np.uint64(cl)).astype(np.int64)], cl, seed)
+            assert bad == 0, (l, bad)
+        a.layer_ready(x, -1, aeg.READY_BLOCK)
+        a.xfer_release(x)
+        assert a.kernel_stats(aeg.K_MIGRATE)[0] == 2     # [0, 2) and [2, 3)
+        bad = 0
+        allo = np.arange(cells, dtype=np.uint64) * np.uint64(cl)
+        for i in range(0, cells, 1 << 16):
+            bd, _ = D.verify_chunks(bbase, allo[i:i + (1 << 16)], exp[i:i + (1 << 16)], cl, seed)
+            bad += bd
+        assert bad == 0
+    finally:
+        a.shutdown()
+        b.shutdown()
+
+
 def test_c4_full_size_three_model_switch():
     """configs[3] at full size: Qwen-1.8B / Llama-7B / Yi-9B weights (3.7 / 13.5 / 17.7 GB, generated
     pageable Model Caches) with 1 GiB of KV each, switched A -> B -> C -> A in the production order
