@@ -625,7 +625,7 @@ def small_chunk_leg(aeg, torch, kernel, model="yi-9b", gib=1):
 
 
 
-def c1_leg(aeg, torch, kernel, reps=200):
+def c1_leg(aeg, torch, kernel, reps=200, pack_mib=0):
     """configs[0] (tiny: 2 layers, 4 KV heads, d=64, fp16, 16-token blocks, 8 requests <= 256
     tokens, 75 blocks, 2.3 MiB) swap round trip: launch/latency-bound, so report the per-round-trip
     latency (GPU: consumer-stream events from the fence to the swap-in's last layer; wall: the two
@@ -645,7 +645,8 @@ def c1_leg(aeg, torch, kernel, reps=200):
                                             dev_slab_bytes=256 * kib, host_slab_bytes=256 * kib,
                                             staging_slot_bytes=8 << 20, staging_slots=2, stage_ring_bytes=2 << 20,
                                             stage_chunk_bytes=1 << 20, device_weight_bytes=2 << 20,
-                                            table_arena_bytes=2 << 20, host_threads=1, kernel=kernel))
+                                            table_arena_bytes=2 << 20, host_threads=1, kernel=kernel,
+                                            pack_layer_mib=pack_mib))
     dbase, _ = ctx.pool_region(0)
     src = ctx.kv_alloc(0, sht, nb)
     keys = np.array([gi.kv_key(1, 0, i, l) for i in range(nb) for l in range(sh.num_layers)], np.uint64)
@@ -2251,7 +2252,15 @@ def run_ours(args):
         else:
             c5 = {"skipped": "configs[4] is the 8-GPU TP=4 layout (one rank pair on 1 GPU); not defined for N=%d" % world}
         small = None if world > 1 else leg("small_chunk", lambda: small_chunk_leg(aeg, torch, kernel))
-        c1 = None if world > 1 else leg("c1", lambda: c1_leg(aeg, torch, kernel))
+        def c1_both():
+            r = c1_leg(aeg, torch, kernel)
+            # the same with one staging segment per layer (pack_layer_mib = 1): the swap-in's H2D of
+            # layer 0 overlaps the swap-out's D2H of layer 1 (duplex), at a few µs more enqueue
+            q = c1_leg(aeg, torch, kernel, pack_mib=1)
+            r["per_layer_segments"] = {k: q[k] for k in ("round_trip_gpu_us_p50", "round_trip_wall_us_p50",
+                                                          "enqueue_us_p50", "bit_exact")}
+            return r
+        c1 = None if world > 1 else leg("c1", c1_both)
         small_tp4 = None if world > 1 else leg("small_chunk_tp4",
                                                lambda: small_chunk_leg(aeg, torch, kernel, model="yi-9b-tp4"))
         route = None if world > 1 else leg("host_route", lambda: host_route_leg(aeg, torch, kernel))
