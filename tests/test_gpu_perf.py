@@ -1,7 +1,8 @@
 """Performance floor (not parity): the gather / scatter kernels of a swap must stay HBM-bound —
 at least 0.70 of the measured copy peak (north star target; they run at ~0.9–0.97), timed by the
 library's own CUDA events (AEG_CFG_TIMING) on 1 GiB per direction (one launch each way), for
-256 KiB (Qwen-7B) and 8 KiB (Yi-9B TP=4 rank) chunks.  PCIe rates are not asserted: they vary by box."""
+256 KiB (Qwen-7B) and 8 KiB (Yi-9B TP=4 rank) chunks.  PCIe rates are not asserted: they vary by box.  Also the local hand-off (fused paged -> paged
+migrate kernel) at the same floor."""
 import json
 import os
 
@@ -50,3 +51,35 @@ def test_swap_kernels_stay_hbm_bound(shape):
             assert gbps >= floor, f"{name}: {gbps:.0f} GB/s < {floor:.0f} (0.70 of the measured copy peak)"
     finally:
         ctx.shutdown()
+
+
+def test_local_hand_off_stays_hbm_bound():
+    """The fused paged -> paged migrate kernel (local hand-off, packed >= ~1 ms launches): at least
+    0.70 of the measured copy peak in HBM traffic (2 x payload) on 4 GiB of Llama-2-13B-shaped
+    blocks from a layer-major pool into a block-major pool of another context (~0.96 measured)."""
+    require_gpu()
+    shape = (40, 40, 128, 2, 16)             # Llama-2-13B: 320 KiB chunks, 12.5 MiB blocks
+    sh = aeg.KVShape.of(shape)
+    n = (4 * GIB) // sh.block_bytes()
+    slab = GIB + (256 << 20)
+    nslab = -(-n // (slab // sh.block_bytes())) + 1
+    mk = lambda lay: aeg.Context(0, aeg.default_config(device_kv_bytes=nslab * slab, host_kv_bytes=GIB,  # noqa: E731
+                                                       dev_slab_bytes=slab, dev_slab_layout=lay,
+                                                       flags=aeg.CFG_TIMING))
+    a, b = mk(aeg.LAYER_MAJOR), mk(aeg.BLOCK_MAJOR)
+    try:
+        src, dst = a.kv_alloc(0, shape, n), b.kv_alloc(0, shape, n)
+        a.import_peer(1, b.export_ipc())
+        for _ in range(3):
+            a.kernel_stats_reset()
+            x = a.kv_migrate(shape, src, 1, dst)
+            a.layer_ready(x, -1, aeg.READY_BLOCK)
+            a.xfer_release(x)
+        launches, nbytes, ms = a.kernel_stats(aeg.K_MIGRATE)
+        assert launches >= 1 and ms > 0
+        gbps = nbytes / (ms * 1e6)
+        floor = 0.70 * _peak()
+        assert gbps >= floor, f"migrate: {gbps:.0f} GB/s < {floor:.0f} (0.70 of the measured copy peak)"
+    finally:
+        a.shutdown()
+        b.shutdown()
