@@ -1,8 +1,8 @@
 """Performance floor (not parity): the gather / scatter kernels of a swap must stay HBM-bound —
 at least 0.70 of the measured copy peak (north star target; they run at ~0.9–0.97), timed by the
 library's own CUDA events (AEG_CFG_TIMING) on 1 GiB per direction (one launch each way), for
-256 KiB (Qwen-7B) and 8 KiB (Yi-9B TP=4 rank) chunks.  PCIe rates are not asserted: they vary by box.  Also the local hand-off (fused paged -> paged
-migrate kernel) at the same floor."""
+256 KiB (Qwen-7B) and 8 KiB (Yi-9B TP=4 rank) chunks; and the local hand-off (fused paged -> paged
+migrate kernel) at the same floor.  PCIe rates are not asserted: they vary by box."""
 import json
 import os
 
