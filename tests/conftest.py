@@ -9,7 +9,7 @@ if ROOT not in sys.path:
 
 # GPU files run cheapest-parity-first, so that under -x a failure in a heavy test (full-size pools,
 # multi-process IPC, race stress) cannot hide the C1 parity results; everything else keeps its order.
-_GPU_ORDER = ["test_gpu_swap.py", "test_gpu_dma_edges.py", "test_c_client.py", "test_gpu_edges.py", "test_gpu_shapes.py", "test_gpu_weights.py",
+_GPU_ORDER = ["test_gpu_swap.py", "test_gpu_dma_edges.py", "test_c_client.py", "test_gpu_edges.py", "test_gpu_fuzz.py", "test_gpu_shapes.py", "test_gpu_weights.py",
               "test_gpu_switch.py", "test_gpu_migrate.py", "test_gpu_dist.py", "test_gpu_stress.py", "test_gpu_c5.py",
               "test_gpu_fullsize.py"]
 

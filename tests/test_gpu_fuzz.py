@@ -1,0 +1,111 @@
+"""Seeded fuzz of the whole swap / hand-off path against the oracle: random KV shapes (chunks from
+32 B to 128 KiB, 1-6 layers), slab sizes with ragged tails, both slab layouts on each side, every
+kernel, layer packing and D2H piece sizes, aged pools; per case a swap-out, a swap-in into fresh
+blocks and a local hand-off (fused kernel or copy-engine route), each compared with O5 / O6 / O7 on
+the whole device and host pool images (every byte, including everything that must stay untouched)."""
+import numpy as np
+import pytest
+
+import aeg_inputs as gi
+import paper_conf_sosp_xiang0qyzyzl0025_b200 as aeg
+from oracle import kv as OK
+from oracle.shape import KVShape
+
+from .gpu_harness import Side, fill_blocks, first_diff, poison_blocks, require_gpu
+
+pytestmark = pytest.mark.gpu
+
+MIB = 1 << 20
+KERNELS = [aeg.KERNEL_AUTO, aeg.KERNEL_LSU, aeg.KERNEL_BULK, aeg.KERNEL_WARP, aeg.KERNEL_BULKW]
+
+
+def draw(seed):
+    """One case: a shape whose chunk is a multiple of 16 B, slab geometry for both pools, config."""
+    r = np.random.default_rng(0xF022 + seed)
+    while True:
+        L, H = int(r.integers(1, 7)), int(r.choice([1, 2, 3, 5, 8]))
+        D, B = int(r.choice([8, 16, 64, 128])), int(r.choice([1, 2, 16, 32]))
+        sh = KVShape(L, H, D, 2, B)
+        if sh.chunk_bytes() % 16 == 0 and sh.block_bytes() <= 2 * MIB:
+            break
+
+    def slab():
+        k = int(r.integers(1, 10))
+        while k > 1 and k * sh.block_bytes() > 6 * MIB:
+            k -= 1
+        tail = 16 * int(r.integers(0, max(1, sh.block_bytes() // 16)))   # ragged tail < one block
+        s = k * sh.block_bytes() + tail
+        return s, max(3, min(12, (16 * MIB) // s))
+    (ds, dn), (hs, hn) = slab(), slab()
+    return dict(sh=sh, dev_slab=ds, dev_slabs=dn, host_slab=hs, host_slabs=hn,
+                dev_layout=int(r.integers(0, 2)), host_layout=int(r.integers(0, 2)),
+                kernel=int(r.choice(KERNELS)), pack=int(r.choice([1, 32])), piece=int(r.choice([1, 128])),
+                ce=bool(r.integers(0, 2)), rng=r)
+
+
+@pytest.mark.parametrize("seed", range(64))
+def test_fuzz_swap_and_hand_off_match_the_oracle(seed):
+    require_gpu()
+    c = draw(seed)
+    sh, r = c["sh"], c["rng"]
+    cfg = aeg.default_config(device_kv_bytes=c["dev_slabs"] * c["dev_slab"],
+                             host_kv_bytes=c["host_slabs"] * c["host_slab"],
+                             dev_slab_bytes=c["dev_slab"], host_slab_bytes=c["host_slab"],
+                             dev_slab_layout=c["dev_layout"], host_slab_layout=c["host_layout"],
+                             staging_slot_bytes=MIB, staging_slots=2, stage_ring_bytes=4 * MIB,
+                             stage_chunk_bytes=MIB, device_weight_bytes=2 * MIB, table_arena_bytes=4 * MIB,
+                             host_threads=1, kernel=c["kernel"], pack_layer_mib=c["pack"],
+                             dma_piece_mib=c["piece"])
+    ctx = aeg.Context(0, cfg)
+    try:
+        dev = Side(ctx, aeg.POOL_DEVICE, cfg.device_kv_bytes, cfg.dev_slab_bytes, c["dev_layout"])
+        host = Side(ctx, aeg.POOL_HOST, cfg.host_kv_bytes, cfg.host_slab_bytes, c["host_layout"])
+        dev.poison(gi.TAG_NEVER)
+        host.poison(gi.TAG_NEVER)
+        dimg, himg = dev.poison_img(gi.TAG_NEVER), host.poison_img(gi.TAG_NEVER)
+        kd = cfg.dev_slab_bytes // sh.block_bytes()
+        kh = cfg.host_slab_bytes // sh.block_bytes()
+        cap_d, cap_h = c["dev_slabs"] * kd, c["host_slabs"] * kh
+        # age the device pool: a few seeded allocations, some freed again
+        live = []
+        for _ in range(int(r.integers(0, 6))):
+            m = int(r.integers(1, max(2, cap_d // 8)))
+            if sum(len(o) for _, o in live) + m > cap_d // 4:
+                break
+            live.append(dev.alloc(sh, m))
+        for i in sorted(r.permutation(len(live))[: len(live) // 2], reverse=True):
+            dev.free(*live.pop(int(i)))
+        used = sum(len(o) for _, o in live)
+        n = int(r.integers(1, max(2, min(cap_h, (cap_d - used) // 3) + 1)))
+        dc, do = dev.alloc(sh, n)
+        fill_blocks(dev, dimg, sh, do, [(0, j) for j in range(n)], m=2)
+        assert first_diff(dev.read(), dimg) is None
+        # swap-out (FREE_SRC: the sources sit in the move list until it completes)
+        hc, ho = host.alloc(sh, n)
+        x = ctx.kv_swap_out(sh.as_tuple(), dc, hc, flags=aeg.FREE_SRC)
+        xo = dev.oracle.begin(do)
+        dev.oracle.free(do)
+        himg = OK.swap_out(dimg, dev.geom, himg, host.geom, sh, do, ho)
+        ctx.layer_ready(x, -1, aeg.READY_BLOCK)
+        assert first_diff(host.read(), himg) is None, c
+        assert first_diff(dev.read(), dimg) is None, c
+        dev.oracle.complete(xo)
+        # swap-in into fresh blocks
+        nc, no = dev.alloc(sh, n)
+        poison_blocks(dev, dimg, sh, no)
+        y = ctx.kv_swap_in(sh.as_tuple(), hc, nc)
+        dimg = OK.swap_in(himg, host.geom, dimg, dev.geom, sh, ho, no)
+        ctx.layer_ready(y, -1, aeg.READY_BLOCK)
+        assert first_diff(dev.read(), dimg) is None, c
+        # local hand-off of the swapped-in blocks into fresh blocks of the same pool
+        mc, mo = dev.alloc(sh, n)
+        poison_blocks(dev, dimg, sh, mo)
+        z = ctx.kv_migrate(sh.as_tuple(), nc, -1, mc, flags=aeg.MIGRATE_CE if c["ce"] else 0)
+        dimg = OK.migrate(dimg, dev.geom, dimg, dev.geom, sh, no, mo)
+        ctx.layer_ready(z, -1, aeg.READY_BLOCK)
+        assert first_diff(dev.read(), dimg) is None, c
+        assert first_diff(host.read(), himg) is None, c
+        for t in (x, y, z):
+            ctx.xfer_release(t)
+    finally:
+        ctx.shutdown()
