@@ -109,3 +109,47 @@ def test_fuzz_swap_and_hand_off_match_the_oracle(seed):
             ctx.xfer_release(t)
     finally:
         ctx.shutdown()
+
+
+@pytest.mark.parametrize("seed", range(32))
+def test_fuzz_hand_off_between_contexts_of_different_geometry(seed):
+    """Prefill context -> decode context of this process (peer mapped directly), each pool with its
+    own random slab size, ragged tail and layout; fused kernel or copy-engine route; the whole
+    destination pool vs O7 and the source pool unchanged."""
+    require_gpu()
+    c = draw(1000 + seed)
+    sh, r = c["sh"], c["rng"]
+
+    def mk(slab, slabs, layout):
+        cfg = aeg.default_config(device_kv_bytes=slabs * slab, host_kv_bytes=MIB, dev_slab_bytes=slab,
+                                 host_slab_bytes=MIB, dev_slab_layout=layout, staging_slot_bytes=MIB,
+                                 staging_slots=2, stage_ring_bytes=4 * MIB, stage_chunk_bytes=MIB,
+                                 device_weight_bytes=2 * MIB, table_arena_bytes=4 * MIB, host_threads=1,
+                                 kernel=c["kernel"])
+        ctx = aeg.Context(0, cfg)
+        return ctx, Side(ctx, aeg.POOL_DEVICE, cfg.device_kv_bytes, slab, layout)
+    a, src = mk(c["dev_slab"], c["dev_slabs"], c["dev_layout"])
+    b, dst = mk(c["host_slab"], c["host_slabs"], c["host_layout"])    # the second geometry of the case
+    try:
+        for s in (src, dst):
+            s.poison(gi.TAG_NEVER)
+        simg, dimg = src.poison_img(gi.TAG_NEVER), dst.poison_img(gi.TAG_NEVER)
+        cap_s = c["dev_slabs"] * (c["dev_slab"] // sh.block_bytes())
+        cap_d = c["host_slabs"] * (c["host_slab"] // sh.block_bytes())
+        if cap_d > 2:   # some resident blocks first, so the destination blocks are not the first ones
+            dst.alloc(sh, int(r.integers(1, cap_d // 2)))
+        n = int(r.integers(1, max(2, min(cap_s, cap_d - dst.oracle.owner_count()) + 1)))
+        sc, so = src.alloc(sh, n)
+        fill_blocks(src, simg, sh, so, [(1, j) for j in range(n)], m=3)
+        dc, do = dst.alloc(sh, n)
+        poison_blocks(dst, dimg, sh, do)
+        a.import_peer(1, b.export_ipc())
+        x = a.kv_migrate(sh.as_tuple(), sc, 1, dc, flags=aeg.MIGRATE_CE if c["ce"] else 0)
+        exp = OK.migrate(simg, src.geom, dimg, dst.geom, sh, so, do)
+        a.layer_ready(x, -1, aeg.READY_BLOCK)
+        assert first_diff(dst.read(), exp) is None, c
+        assert first_diff(src.read(), simg) is None, c
+        a.xfer_release(x)
+    finally:
+        a.shutdown()
+        b.shutdown()
