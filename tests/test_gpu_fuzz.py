@@ -1,4 +1,4 @@
-"""Seeded fuzz of the whole swap / hand-off path against the oracle: random KV shapes (chunks from
+"""Seeded fuzz of the whole swap / hand-off path (and weight staging, last test) against the oracle: random KV shapes (chunks from
 32 B to 128 KiB, 1-6 layers), slab sizes with ragged tails, both slab layouts on each side, every
 kernel, layer packing and D2H piece sizes, aged pools; per case a swap-out, a swap-in into fresh
 blocks and a local hand-off (fused kernel or copy-engine route), each compared with O5 / O6 / O7 on
@@ -153,3 +153,65 @@ def test_fuzz_hand_off_between_contexts_of_different_geometry(seed):
     finally:
         a.shutdown()
         b.shutdown()
+
+
+@pytest.mark.parametrize("seed", range(24))
+def test_fuzz_weight_staging_matches_the_oracle(seed):
+    """Random tensor lists (REPLICATED / COL with 1 or 3 groups / ROW / VOCAB splits, odd sizes),
+    TP size and rank, Stage Buffer chunk / ring / thread counts, staged or registered-direct path,
+    two jobs back to back (the second bumps on from the first): the weights region vs oracle O8."""
+    require_gpu()
+    from aeg_inputs import dev as D
+    from oracle import weights as W
+    r = np.random.default_rng(0x3E16 + seed)
+    tp = int(r.choice([1, 2, 3, 4, 8]))
+    rank = int(r.integers(0, tp))
+
+    def tensors(m):
+        descs = []
+        for k in range(int(r.integers(1, 10))):
+            split = int(r.choice([W.REPLICATED, W.COL, W.ROW, W.VOCAB]))
+            groups = int(r.choice([1, 3])) if split == W.COL else 1
+            rows = int(r.integers(1, 64)) * (groups * tp if split in (W.COL, W.VOCAB) else 1)
+            cols = int(r.integers(1, 300)) * (tp if split == W.ROW else 1)
+            descs.append(dict(rows=rows, cols=cols, split=split, groups=groups, layer=int(r.integers(0, 4))))
+        sizes = [d["rows"] * d["cols"] * 2 for d in descs]
+        buf = np.empty(sum(-(-n // 256) * 256 for n in sizes) + 256, np.uint8)
+        tens, o = [], 0
+        for k, (d, n) in enumerate(zip(descs, sizes)):
+            v = buf[o:o + n]
+            v[:] = gi.region_bytes(gi.w_seed(9), gi.weight_key(m, k), n)
+            tens.append(v.reshape(d["rows"], d["cols"] * 2))
+            o += -(-n // 256) * 256
+        return descs, buf, tens
+    direct = bool(r.integers(0, 2))
+    chunk = int(r.choice([1, 2, 4])) << 20
+    cfg = aeg.default_config(device_kv_bytes=4 * MIB, host_kv_bytes=4 * MIB, dev_slab_bytes=MIB,
+                             host_slab_bytes=MIB, stage_ring_bytes=chunk * int(r.integers(2, 5)),
+                             stage_chunk_bytes=chunk, staging_slot_bytes=MIB, staging_slots=2,
+                             device_weight_bytes=48 * MIB, table_arena_bytes=2 * MIB,
+                             host_threads=int(r.integers(1, 5)))
+    ctx = aeg.Context(0, cfg)
+    try:
+        base, wbytes, _ = ctx.weights_region()
+        exp, end, shards = None, 0, []
+        for m in (1, 2):
+            descs, buf, tens = tensors(m)
+            if direct:
+                ctx.host_register(buf.ctypes.data, buf.nbytes)
+            dl = [dict(host_src=t.ctypes.data, rows=d["rows"], cols=d["cols"], elem_bytes=2, layer=d["layer"],
+                       split=d["split"], groups=d["groups"]) for t, d in zip(tens, descs)]
+            offs, x = ctx.weights_stage(dl, tp_rank=rank, tp_size=tp)
+            ctx.layer_ready(x, -1, aeg.READY_BLOCK)
+            exp, eoffs, end = W.stage(tens, descs, rank, tp, region_bytes=wbytes, base=end, dst=exp)
+            assert [int(o) for o in offs] == eoffs
+            shards += [(o, W.shard(t.reshape(d["rows"], d["cols"], 2), d["split"], d["groups"], rank, tp).size)
+                       for o, t, d in zip(eoffs, tens, descs)]
+            got = D.read(base, end)
+            for o, n in shards:   # every shard of both jobs (padding between shards is unspecified)
+                assert first_diff(got[o:o + n], exp[o:o + n]) is None, (seed, m, tp, rank, direct, o)
+            ctx.xfer_release(x)
+            if direct:
+                ctx.host_unregister(buf.ctypes.data)
+    finally:
+        ctx.shutdown()
