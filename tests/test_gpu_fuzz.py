@@ -1,8 +1,9 @@
-"""Seeded fuzz of the whole swap / hand-off path (and weight staging, last test) against the oracle: random KV shapes (chunks from
-32 B to 128 KiB, 1-6 layers), slab sizes with ragged tails, both slab layouts on each side, every
-kernel, layer packing and D2H piece sizes, aged pools; per case a swap-out, a swap-in into fresh
-blocks and a local hand-off (fused kernel or copy-engine route), each compared with O5 / O6 / O7 on
-the whole device and host pool images (every byte, including everything that must stay untouched)."""
+"""Seeded fuzz against the oracle.  Swap / hand-off: random KV shapes (chunks from 32 B to 128 KiB,
+1-6 layers), slab sizes with ragged tails, both slab layouts on each side, every kernel, layer
+packing and D2H piece sizes, aged pools; per case a swap-out, a swap-in into fresh blocks and a local
+hand-off (fused kernel or copy-engine route), each compared with O5 / O6 / O7 on the whole device and
+host pool images (every byte, including everything that must stay untouched); hand-offs between
+contexts of different pool geometry (O7); and weight staging with random splits (O8)."""
 import numpy as np
 import pytest
 
