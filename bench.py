@@ -638,9 +638,10 @@ def c1_leg(aeg, torch, kernel, reps=200, pack_mib=0):
     lens = gi.request_lengths(1, 8, 1, 256, forced=(1, 16, 17, 255, 256))
     nb = sum(-(-t // 16) for t in lens)
     kib = 1024
-    # staging slots of 8 MiB: the whole 2.3 MiB batch (both layers) is one segment, i.e. one gather /
-    # scatter launch and one copy per host run (1 MiB slots cut each layer in two: 4 segments and
-    # ~2x the enqueue time, tools/enqueue_probe.py)
+    # staging slots of 8 MiB: one segment per layer (the planner keeps >= 4 segments, so a 2-layer
+    # transfer is never packed into one: the swap-in's H2D of layer 0 overlaps the swap-out's D2H of
+    # layer 1 — 147 vs 172 us as one packed segment); 1 MiB slots would cut each layer in two (more
+    # segments, ~2x the enqueue time, tools/enqueue_probe.py)
     ctx = aeg.Context(0, aeg.default_config(device_kv_bytes=32 * 256 * kib, host_kv_bytes=32 * 256 * kib,
                                             dev_slab_bytes=256 * kib, host_slab_bytes=256 * kib,
                                             staging_slot_bytes=8 << 20, staging_slots=2, stage_ring_bytes=2 << 20,
@@ -1815,18 +1816,25 @@ def kernel_alone_leg(aeg, kernel, shape=None):
     return out
 
 
-def kernel_alone_once(aeg, kernel, shape=None, spread_gib=16):
-    """The dominant kernels without the step's concurrent PCIe DMA: one 1 GiB swap-out and swap-in of
-    the C2 shape with every layer in one staging segment (pack_layer_mib = 1024), i.e. one gather and
-    one scatter launch, timed by the library's CUDA events (AEG_CFG_TIMING); best of 3.  The blocks
-    are paged like the step's: a seeded random 1 GiB of blocks kept out of a spread_gib pool that was
-    filled and then mostly freed, so both kernels walk block tables spread over the whole pool."""
+# one layer of Qwen-7B-sized chunks (256 KiB): 4,096 blocks are one 1 GiB staging segment, i.e. one
+# gather and one scatter launch — the step's launch size (3,970 x 256 KiB) — with no copy-engine DMA
+# running during either kernel (the D2H starts after the gather, the scatter after the H2D)
+ALONE_SHAPE = (1, 32, 128, 2, 16)
+
+
+def kernel_alone_once(aeg, kernel, shape=None, spread_gib=16, layer_gib=1):
+    """The dominant kernels without the step's concurrent PCIe DMA: a swap-out and a swap-in of one
+    layer of layer_gib (one gather and one scatter launch of the step's size), timed by the library's
+    CUDA events (AEG_CFG_TIMING); best of 3.  The blocks are paged like the step's: a
+    seeded random set kept out of a spread_gib pool that was filled and then mostly freed, so both
+    kernels walk block tables spread over the whole pool (spread_gib = 0: the contiguous best case)."""
     import aeg_inputs as gi
-    shape = shape or QWEN7B
+    shape = shape or ALONE_SHAPE
     sh = aeg.KVShape.of(shape)
-    n = GIB // sh.block_bytes()
-    ctx = aeg.Context(0, aeg.default_config(device_kv_bytes=max(spread_gib, 4) * GIB, host_kv_bytes=2 * GIB,
-                                            pack_layer_mib=1024, kernel=kernel, flags=aeg.CFG_TIMING))
+    n = (layer_gib * GIB) // sh.chunk_bytes()
+    total = n * sh.block_bytes()
+    ctx = aeg.Context(0, aeg.default_config(device_kv_bytes=max(spread_gib * GIB, total + GIB),
+                                            host_kv_bytes=total + GIB, kernel=kernel, flags=aeg.CFG_TIMING))
     best = {}
     try:
         if spread_gib:
@@ -2252,15 +2260,7 @@ def run_ours(args):
         else:
             c5 = {"skipped": "configs[4] is the 8-GPU TP=4 layout (one rank pair on 1 GPU); not defined for N=%d" % world}
         small = None if world > 1 else leg("small_chunk", lambda: small_chunk_leg(aeg, torch, kernel))
-        def c1_both():
-            r = c1_leg(aeg, torch, kernel)
-            # the same with one staging segment per layer (pack_layer_mib = 1): the swap-in's H2D of
-            # layer 0 overlaps the swap-out's D2H of layer 1 (duplex), at a few µs more enqueue
-            q = c1_leg(aeg, torch, kernel, pack_mib=1)
-            r["per_layer_segments"] = {k: q[k] for k in ("round_trip_gpu_us_p50", "round_trip_wall_us_p50",
-                                                          "enqueue_us_p50", "bit_exact")}
-            return r
-        c1 = None if world > 1 else leg("c1", c1_both)
+        c1 = None if world > 1 else leg("c1", lambda: c1_leg(aeg, torch, kernel))
         small_tp4 = None if world > 1 else leg("small_chunk_tp4",
                                                lambda: small_chunk_leg(aeg, torch, kernel, model="yi-9b-tp4"))
         route = None if world > 1 else leg("host_route", lambda: host_route_leg(aeg, torch, kernel))

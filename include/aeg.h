@@ -133,7 +133,8 @@ typedef struct {
                                    blocks until the copy engine drains (correct, not async)      */
   uint32_t pack_layer_mib;      /* KV swaps: layers smaller than this share one staging segment
                                    (one kernel launch, fewer copy commands, readiness per
-                                   segment); 0 = the default                      */
+                                   segment), keeping >= 4 segments per transfer (fewer layers:
+                                   one per segment); 0 = the default             */
   uint32_t reserved[4];
 } aeg_config;
 

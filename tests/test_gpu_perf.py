@@ -1,7 +1,7 @@
 """Performance floor (not parity): the gather / scatter kernels of a swap must stay HBM-bound —
 at least 0.70 of the measured copy peak (north star target; they run at ~0.9–0.97), timed by the
-library's own CUDA events (AEG_CFG_TIMING) on 1 GiB per direction (one launch each way), for
-256 KiB (Qwen-7B) and 8 KiB (Yi-9B TP=4 rank) chunks; and the local hand-off (fused paged -> paged
+library's own CUDA events (AEG_CFG_TIMING) on one 1 GiB launch each way (the bench step's launch
+size), for 256 KiB (Qwen-7B) and 8 KiB (Yi-9B TP=4 rank) chunks; and the local hand-off (fused paged -> paged
 migrate kernel) at the same floor.  PCIe rates are not asserted: they vary by box."""
 import json
 import os
@@ -22,15 +22,15 @@ def _peak():
     return float(json.load(open(p))["hbm_gbs"]) if os.path.exists(p) else 6650.0
 
 
-@pytest.mark.parametrize("shape", [(32, 32, 128, 2, 16), (48, 1, 128, 2, 16)], ids=["256KiB", "8KiB"])
+@pytest.mark.parametrize("shape", [(1, 32, 128, 2, 16), (1, 1, 128, 2, 16)], ids=["256KiB", "8KiB"])
 def test_swap_kernels_stay_hbm_bound(shape):
     require_gpu()
     sh = aeg.KVShape.of(shape)
-    n = GIB // sh.block_bytes()
-    # pack every layer into one 1 GiB segment: one gather and one scatter launch per transfer, so the
-    # events time the kernel body rather than per-launch overhead
-    ctx = aeg.Context(0, aeg.default_config(device_kv_bytes=4 * GIB, host_kv_bytes=2 * GIB,
-                                            pack_layer_mib=1024, flags=aeg.CFG_TIMING))
+    n = GIB // sh.chunk_bytes()          # one 1 GiB layer = one staging segment: one launch each way,
+                                         # with no copy-engine DMA running during either kernel
+    total = n * sh.block_bytes()
+    ctx = aeg.Context(0, aeg.default_config(device_kv_bytes=total + GIB, host_kv_bytes=total + GIB,
+                                            flags=aeg.CFG_TIMING))
     try:
         dev = ctx.kv_alloc(aeg.POOL_DEVICE, shape, n)
         for _ in range(3):   # warm-up rounds, then measure the last
@@ -46,7 +46,7 @@ def test_swap_kernels_stay_hbm_bound(shape):
         floor = 0.70 * _peak()
         for kind, name in ((aeg.K_GATHER, "gather"), (aeg.K_SCATTER, "scatter")):
             launches, nbytes, ms = ctx.kernel_stats(kind)
-            assert launches > 0 and ms > 0
+            assert launches == sh.num_layers and ms > 0
             gbps = nbytes / (ms * 1e6)
             assert gbps >= floor, f"{name}: {gbps:.0f} GB/s < {floor:.0f} (0.70 of the measured copy peak)"
     finally:
