@@ -57,6 +57,24 @@ def test_random_overlapping_transfers_with_d2h_pieces(seed):
     assert n_out > 0 and sum(1 for e in log if e[0] == "op" and e[1] == "d2h") > n_out * SHB.L
 
 
+SHP = KVShape(8, 2, 64, 2, 16)           # 8 KiB chunks, 8 layers: small layers are packed 2 per segment
+
+
+@pytest.mark.parametrize("seed", range(4))
+def test_random_overlapping_transfers_with_packed_layers(seed):
+    """The same stress with layers small enough to be packed (default pack_layer_mib; the planner
+    keeps >= 4 segments, so 2 of the 8 layers share each segment): per-layer events recorded after a
+    multi-layer segment, waited for per layer by later transfers."""
+    cfg = aeg.default_config(device_kv_bytes=24 * 512 * KIB, host_kv_bytes=24 * 512 * KIB, dev_slab_bytes=512 * KIB,
+                             host_slab_bytes=512 * KIB, dev_slab_layout=seed % 2, host_slab_layout=(seed // 2) % 2,
+                             staging_slot_bytes=1 << 20, staging_slots=2, stage_ring_bytes=4 << 20,
+                             stage_chunk_bytes=1 << 20, device_weight_bytes=2 << 20, table_arena_bytes=2 << 20,
+                             host_threads=1, kernel=aeg.KERNEL_AUTO)
+    log, _ = _stress(200 + seed, cfg, SHP, 12)
+    # packing really happened: some gather read two layers in one segment
+    assert any(e[0] == "op" and e[1] == "gather" and len({c.rsplit(":", 1)[1] for c in e[3]}) == 2 for e in log)
+
+
 def _stress(seed, cfg, SH, nmax, lo=1):
     require_gpu()
     import torch
