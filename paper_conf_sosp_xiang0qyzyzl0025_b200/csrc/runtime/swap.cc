@@ -14,6 +14,12 @@
 
 #include "engine.h"
 
+// Layers per local hand-off launch, in MiB (see Ctx::migrate); overridable for experiments
+// (tools/gpu_migrate_pack.sh builds with -DAEG_MIGRATE_LOCAL_PACK_MIB=...).
+#ifndef AEG_MIGRATE_LOCAL_PACK_MIB
+#define AEG_MIGRATE_LOCAL_PACK_MIB 4096
+#endif
+
 namespace aeg {
 
 namespace {
@@ -691,9 +697,6 @@ uint64_t Ctx::migrate(const Shape& sh, const aeg_block* src, int32_t peer, const
   // to >= ~1 ms of copying per launch: 4 GiB on the same GPU (HBM speed), 512 MiB over NVLink
   // (~0.7 ms at the measured 770 GB/s peer copy).  Every layer still gets its event, recorded when
   // its launch completes; layers larger than the pack go one per launch.
-#ifndef AEG_MIGRATE_LOCAL_PACK_MIB  // overridable for experiments (tools/gpu_migrate_pack.sh)
-#define AEG_MIGRATE_LOCAL_PACK_MIB 4096
-#endif
   const bool remote = P && (!P->same_process || P->device != device);
   const uint64_t pack = remote ? (512ull << 20) : (uint64_t(AEG_MIGRATE_LOCAL_PACK_MIB) << 20);
   const uint64_t layer = uint64_t(n) * sh.chunk();
