@@ -171,6 +171,32 @@ __device__ __forceinline__ void bulk_store(void* gdst, const void* ssrc, uint32_
   asm volatile("cp.async.bulk.commit_group;" ::: "memory");
 }
 
+#ifdef AEG_BW_EVICT_FIRST  // experiment: streaming L2 policy on the BULKW bulk copies
+__device__ __forceinline__ uint64_t evict_first_policy() {
+  uint64_t pol;
+  asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(pol));
+  return pol;
+}
+
+__device__ __forceinline__ void bulk_load_ef(void* sdst, const void* gsrc, uint32_t bytes, uint64_t* bar,
+                                             uint64_t pol) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(bytes)
+               : "memory");
+  asm volatile(
+      "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes.L2::cache_hint [%0], [%1], %2, [%3], %4;" ::"r"(
+          smem_u32(sdst)),
+      "l"(gsrc), "r"(bytes), "r"(smem_u32(bar)), "l"(pol)
+      : "memory");
+}
+
+__device__ __forceinline__ void bulk_store_ef(void* gdst, const void* ssrc, uint32_t bytes, uint64_t pol) {
+  asm volatile("cp.async.bulk.global.shared::cta.bulk_group.L2::cache_hint [%0], [%1], %2, %3;" ::"l"(gdst),
+               "r"(smem_u32(ssrc)), "r"(bytes), "l"(pol)
+               : "memory");
+  asm volatile("cp.async.bulk.commit_group;" ::: "memory");
+}
+#endif
+
 template <int N>
 __device__ __forceinline__ void bulk_wait_read() {
   asm volatile("cp.async.bulk.wait_group.read %0;" ::"n"(N) : "memory");
@@ -280,6 +306,9 @@ __global__ void __launch_bounds__(kBwWarps * 32) copy_bulkw(const CopyArgs a, ui
     const uint64_t rem = a.chunk - off;
     nb = rem < piece ? uint32_t(rem) : piece;
   };
+#ifdef AEG_BW_EVICT_FIRST
+  const uint64_t pol = evict_first_policy();
+#endif
   const char* ls = nullptr;
   char* sd = nullptr;
   uint32_t lnb = 0, snb = 0;
@@ -294,7 +323,11 @@ __global__ void __launch_bounds__(kBwWarps * 32) copy_bulkw(const CopyArgs a, ui
     const char* s = reinterpret_cast<const char*>(
         __shfl_sync(0xffffffffu, reinterpret_cast<unsigned long long>(ls), int(j & 31)));
     const uint32_t nb = __shfl_sync(0xffffffffu, lnb, int(j & 31));
+#ifdef AEG_BW_EVICT_FIRST
+    if (lane == 0) bulk_load_ef(ring + uint64_t(st) * piece, s, nb, &wb[st], pol);
+#else
     if (lane == 0) bulk_load(ring + uint64_t(st) * piece, s, nb, &wb[st]);
+#endif
   };
   auto store = [&](uint64_t j, uint32_t st) {
     if ((j >> 5) != sbatch) {
@@ -305,7 +338,11 @@ __global__ void __launch_bounds__(kBwWarps * 32) copy_bulkw(const CopyArgs a, ui
     }
     char* d = reinterpret_cast<char*>(__shfl_sync(0xffffffffu, reinterpret_cast<unsigned long long>(sd), int(j & 31)));
     const uint32_t nb = __shfl_sync(0xffffffffu, snb, int(j & 31));
+#ifdef AEG_BW_EVICT_FIRST
+    if (lane == 0) bulk_store_ef(d, ring + uint64_t(st) * piece, nb, pol);
+#else
     if (lane == 0) bulk_store(d, ring + uint64_t(st) * piece, nb);
+#endif
   };
   for (uint64_t j = 0; j < mine && j < stages; ++j) load(j, uint32_t(j));
   uint32_t st = 0, phase = 0, prev = stages - 1;
