@@ -400,7 +400,7 @@ uint64_t Ctx::weights_stage(const aeg_weight_desc* d, int32_t n, int32_t r, int3
               (unsigned long long)p, (unsigned long long)cfg.device_weight_bytes);
   std::copy(j->off.begin(), j->off.end(), offs);
   j->start = w_bump;
-  j->end = n > 0 ? j->off.back() + j->size.back() : w_bump;
+  j->end = p;  // through the last shard's 256-byte padding: every padding byte is written (zeros, reading 17)
   j->direct = direct;
   w_bump = p;
   Xfer* x = new_xfer(X_WEIGHTS, L, false);

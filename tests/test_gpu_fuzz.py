@@ -160,7 +160,8 @@ def test_fuzz_hand_off_between_contexts_of_different_geometry(seed):
 def test_fuzz_weight_staging_matches_the_oracle(seed):
     """Random tensor lists (REPLICATED / COL with 1 or 3 groups / ROW / VOCAB splits, odd sizes),
     TP size and rank, Stage Buffer chunk / ring / thread counts, staged or registered-direct path,
-    two jobs back to back (the second bumps on from the first): the weights region vs oracle O8."""
+    two jobs back to back (the second bumps on from the first), over a region holding garbage: every
+    shard vs oracle O8 and every padding byte zero (reading 17)."""
     require_gpu()
     from aeg_inputs import dev as D
     from oracle import weights as W
@@ -195,6 +196,7 @@ def test_fuzz_weight_staging_matches_the_oracle(seed):
     ctx = aeg.Context(0, cfg)
     try:
         base, wbytes, _ = ctx.weights_region()
+        D.fill_region(base, wbytes, gi.w_seed(9), gi.poison_key(gi.TAG_NEVER, 0))   # garbage in the region
         exp, end, shards = None, 0, []
         for m in (1, 2):
             descs, buf, tens = tensors(m)
@@ -209,8 +211,11 @@ def test_fuzz_weight_staging_matches_the_oracle(seed):
             shards += [(o, W.shard(t.reshape(d["rows"], d["cols"], 2), d["split"], d["groups"], rank, tp).size)
                        for o, t, d in zip(eoffs, tens, descs)]
             got = D.read(base, end)
-            for o, n in shards:   # every shard of both jobs (padding between shards is unspecified)
+            for o, n in shards:   # every shard of both jobs
                 assert first_diff(got[o:o + n], exp[o:o + n]) is None, (seed, m, tp, rank, direct, o)
+            # reading 17: the 256-byte padding after every shard (up to the bump pointer) is zeros
+            for (o, n), nxt in zip(shards, [o2 for o2, _ in shards[1:]] + [end]):
+                assert not got[o + n:nxt].any(), (seed, m, tp, rank, direct, o + n, nxt)
             ctx.xfer_release(x)
             if direct:
                 ctx.host_unregister(buf.ctypes.data)
