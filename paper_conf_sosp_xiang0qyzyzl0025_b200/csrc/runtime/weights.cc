@@ -242,7 +242,7 @@ struct WeightPipe {
                                        part_rows * row, cudaMemcpyHostToDevice, s));
           }
           const uint64_t te = j->off[k] + j->size[k];
-          const uint64_t next = k + 1 < j->d.size() ? j->off[k + 1] : align_up(te, 256);
+          const uint64_t next = k + 1 < j->d.size() ? j->off[k + 1] : std::min(j->end, align_up(te, 256));
           if (next > te) CUDA_TRY(cudaMemsetAsync(c->dev_w + te, 0, next - te, s));
           record_layers(j, layer_last, te, s);
         }
@@ -396,11 +396,14 @@ uint64_t Ctx::weights_stage(const aeg_weight_desc* d, int32_t n, int32_t r, int3
       if (s >= rg.first && s + all <= rg.first + rg.second) reg = true;
     direct = direct && reg;
   }
-  AEG_REQUIRE(p <= cfg.device_weight_bytes, AEG_ERR_OOM, "weights region exhausted: need %llu of %llu bytes",
-              (unsigned long long)p, (unsigned long long)cfg.device_weight_bytes);
+  // the region must hold the shards, [start, off_last + size_last) (reading 17, oracle O8); the
+  // padding after the last shard is written only up to the region's end
+  const uint64_t data_end = n > 0 ? j->off.back() + j->size.back() : w_bump;
+  AEG_REQUIRE(data_end <= cfg.device_weight_bytes, AEG_ERR_OOM, "weights region exhausted: need %llu of %llu bytes",
+              (unsigned long long)data_end, (unsigned long long)cfg.device_weight_bytes);
   std::copy(j->off.begin(), j->off.end(), offs);
   j->start = w_bump;
-  j->end = p;  // through the last shard's 256-byte padding: every padding byte is written (zeros, reading 17)
+  j->end = std::min(p, cfg.device_weight_bytes);  // through the last shard's padding (zeros, reading 17)
   j->direct = direct;
   w_bump = p;
   Xfer* x = new_xfer(X_WEIGHTS, L, false);

@@ -151,3 +151,39 @@ def test_invalid_and_oom():
         assert e.value.code == aeg.ERR_OOM
     finally:
         ctx.shutdown()
+
+
+@pytest.mark.parametrize("direct", [False, True])
+def test_region_boundary_matches_the_oracle(direct):
+    """The region must hold the shards, [0, off_last + size_last) (oracle O8, reading 17): with a
+    region size that is not a multiple of the 256-byte bump alignment, an exact fit stages (padding
+    written only up to the region's end), one byte short is ERR_OOM — as in oracle/weights.stage."""
+    require_gpu()
+    descs = [dict(rows=3, cols=100, split=W.REPLICATED, groups=1, layer=0),
+             dict(rows=1, cols=50, split=W.REPLICATED, groups=1, layer=1)]
+    buf, tens = model_cache(descs, m=3)
+    need = 768 + 100                       # 600 B at 0, 100 B at 768 (bump alignment 256)
+    for wbytes, ok in ((need, True), (need - 1, False)):
+        ctx = make(wbytes=wbytes)
+        try:
+            if direct:
+                ctx.host_register(buf.ctypes.data, buf.nbytes)
+            dl = descs_for(tens, descs)
+            if not ok:
+                with pytest.raises(aeg.AegError) as e:
+                    ctx.weights_stage(dl)
+                assert e.value.code == aeg.ERR_OOM
+                with pytest.raises(W.WeightError):
+                    W.stage(tens, descs, 0, 1, region_bytes=wbytes)
+                continue
+            base, _, _ = ctx.weights_region()
+            offs, x = ctx.weights_stage(dl)
+            ctx.layer_ready(x, -1, aeg.READY_BLOCK)
+            exp, eoffs, _ = W.stage(tens, descs, 0, 1, region_bytes=wbytes)
+            assert [int(o) for o in offs] == eoffs == [0, 768]
+            assert first_diff(D.read(base, wbytes), exp[:wbytes]) is None
+            ctx.xfer_release(x)
+            if direct:
+                ctx.host_unregister(buf.ctypes.data)
+        finally:
+            ctx.shutdown()

@@ -126,4 +126,18 @@ def test_stage_leaves_the_given_image_untouched():
     keep = before.copy()
     out, offs, _ = W.stage(ts, descs, 0, 1, 4096, dst=before)
     assert np.array_equal(before, keep)
-    assert np.array_equal(out[:64], ts[0].reshape(-1)) and np.all(out[64:] == 0xAB)
+    assert np.array_equal(out[:64], ts[0].reshape(-1)) and not out[64:256].any() and np.all(out[256:] == 0xAB)
+
+
+def test_padding_after_every_shard_is_zero():
+    """Reading 17: shards sit at 256-byte bump offsets and the padding up to the next
+    offset (and after the last shard, up to the bump pointer) is written as zeros, whatever the
+    region held before; bytes beyond the bump pointer are untouched."""
+    descs = [dict(rows=3, cols=5, split=W.REPLICATED, groups=1), dict(rows=1, cols=7, split=W.REPLICATED, groups=1)]
+    ts = [tensor(3, 5, 11), tensor(1, 7, 12)]
+    before = np.full(2048, 0xCD, np.uint8)
+    out, offs, end = W.stage(ts, descs, 0, 1, 2048, base=256, dst=before)
+    assert offs == [256, 512] and end == 768                   # 30 B -> next at 512; 14 B -> bump 768
+    assert np.array_equal(out[256:286], ts[0].reshape(-1)) and not out[286:512].any()
+    assert np.array_equal(out[512:526], ts[1].reshape(-1)) and not out[526:768].any()
+    assert np.all(out[:256] == 0xCD) and np.all(out[768:] == 0xCD)
